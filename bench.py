@@ -1,0 +1,363 @@
+#!/usr/bin/env python
+"""Benchmark: batched SS-HOPM (solve + dedup [+ NCCL gather]) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+
+A step is one pass of the whole hot path over one batch: sshopm_solve over
+N tensors x S starts, then sshopm_dedup (and, for world size > 1, one NCCL
+gather of the fixed-size dedup records to rank 0).  Inputs are resident in
+HBM before timing starts; L2 is flushed between timed steps (a 512 MiB write
+outside the timed events).  Each rank owns a contiguous tensor range of size
+config N (weak scaling); time = max over ranks of the summed per-step CUDA
+event durations.  Rank 0 prints ONE JSON line.
+
+value = paper-style GFLOP/s = F_paper(m, n) * sum(iters) / time (reading R12,
+SURVEY.md 8(d); lambda_0 excluded).  voxel-solves/s is reported beside it.
+roofline: the solve kernel against the FP32 ALU peak
+148 SM x 128 lanes x 2 flop x f_max, counting the library's
+algorithmic FP32 flops per update (sshopm_flops_per_iter "executed").
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synthetic as syn  # noqa: E402
+
+METRIC = "SS-HOPM Gflop/s & voxel-solves/s (m=4,n=3,128 starts) vs FP32 peak"
+LAM_TOL, ANG_TOL, KMAX = 1e-2, 0.05, 4
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2", choices=sorted(syn.CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--voxels", type=int, default=0, help="override tensors per rank")
+    ap.add_argument("--refill", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-voxels", type=int, default=0)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks --
+class ClockSampler:
+    """NVML SM-clock / throttle-reason sampler running during the timed region."""
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, index, period=0.05):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.period = period
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+        self._stop = threading.Event()
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h) if hasattr(nv, "nvmlDeviceGetCurrentClocksEventReasons") \
+                    else nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name not in ("gpu_idle",):
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def peaks():
+    p = {}
+    f = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(f):
+        with open(f) as fh:
+            p = json.load(fh)
+    return p
+
+
+# --------------------------------------------------------------- CPU oracle --
+def _oracle_chunk(args):
+    cfg, first, count, seed = args
+    from oracle import sshopm as O
+    ent = syn.gen_voxels(cfg["m"], cfg["n"], first, count, seed)
+    st = syn.gen_starts(cfg["S"], cfg["n"], seed)
+    lam, x, it, cv = O.sshopm(ent, st, cfg["m"], cfg["n"], cfg["alpha"], cfg["tol"], cfg["maxit"])
+    return int(it.sum()), count
+
+
+def cpu_oracle(cfg, n_voxels, seed=0, first=0):
+    """Time the FP64 oracle as it stands on the host cores (process pool, one process per core)."""
+    import multiprocessing as mp
+    from oracle.sshopm import paper_flops_per_iter
+    cores = len(os.sched_getaffinity(0))
+    chunk = 64 if cfg["m"] <= 4 and cfg["n"] <= 3 else 16
+    tasks = [(cfg, first + v, min(chunk, n_voxels - v), seed) for v in range(0, n_voxels, chunk)]
+    ctx = mp.get_context("fork")
+    t0 = time.perf_counter()
+    with ctx.Pool(cores) as pool:
+        res = pool.map(_oracle_chunk, tasks, chunksize=1)
+    dt = time.perf_counter() - t0
+    iters = sum(r[0] for r in res)
+    F = paper_flops_per_iter(cfg["m"], cfg["n"])
+    return {"gflops": F * iters / dt / 1e9, "voxel_solves_per_s": n_voxels / dt, "seconds": dt, "cores": cores,
+            "iters": iters, "voxels": n_voxels}
+
+
+def reference_arm(a, cfg, rank, world):
+    """--impl reference: the oracle (FP64 CPU) timed on host cores, rank 0 only."""
+    if rank != 0:
+        return
+    nvox = a.cpu_voxels or (16384 if (cfg["m"], cfg["n"]) == (4, 3) else 1024)
+    for _ in range(a.warmup):
+        cpu_oracle(cfg, min(nvox, 256))
+    tot_t, tot_it, tot_v = 0.0, 0, 0
+    cores = None
+    for s in range(a.steps):
+        r = cpu_oracle(cfg, nvox, seed=0, first=s * nvox)
+        tot_t += r["seconds"]
+        tot_it += r["iters"]
+        tot_v += r["voxels"]
+        cores = r["cores"]
+    from oracle.sshopm import paper_flops_per_iter
+    F = paper_flops_per_iter(cfg["m"], cfg["n"])
+    val = F * tot_it / tot_t / 1e9
+    sample = f"{nvox} tensors x {cfg['S']} starts per step (of {cfg['N']}), FP64 full-tensor numpy oracle, process pool"
+    line = {"metric": METRIC, "value": val, "unit": "GFLOP/s", "impl": "reference", "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * tot_t / a.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": a.config, "m": cfg["m"], "n": cfg["n"], "tensors": cfg["N"], "starts": cfg["S"],
+                       "alpha": cfg["alpha"], "tol": cfg["tol"], "maxit": cfg["maxit"]},
+            "voxel_solves_per_s": tot_v / tot_t,
+            "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- our arm --
+def main():
+    a = parse()
+    cfg = dict(syn.CONFIGS[a.config])
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if a.voxels:
+        cfg["N"] = a.voxels
+    if a.impl == "reference":
+        return reference_arm(a, cfg, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_ballardkp11_b200 as sh
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    m, n, S, Nloc = cfg["m"], cfg["n"], cfg["S"], cfg["N"]
+    solver = sh.Solver(m, n)
+    U = solver.U
+
+    # inputs: this rank's tensor range (counter-based generator -> shard invariant), resident in HBM
+    ent_h = syn.gen_voxels(m, n, rank * Nloc, Nloc, seed=0)
+    st_h = syn.gen_starts(S, n, seed=0)
+    ent = torch.from_numpy(ent_h).to(dev)
+    st = torch.from_numpy(st_h).to(dev)
+    lam = torch.empty((Nloc, S), dtype=torch.float32, device=dev)
+    xo = torch.empty((Nloc, S, n), dtype=torch.float32, device=dev)
+    it = torch.empty((Nloc, S), dtype=torch.int32, device=dev)
+    cv = torch.empty((Nloc, S), dtype=torch.uint8, device=dev)
+    # dedup records packed in one buffer so a single collective moves them
+    rec_words = Nloc * (1 + KMAX * (n + 3))
+    rec = torch.empty(rec_words, dtype=torch.int32, device=dev)
+    o = 0
+    views = []
+    for shape, dt in [((Nloc,), torch.int32), ((Nloc, KMAX), torch.float32), ((Nloc, KMAX, n), torch.float32),
+                      ((Nloc, KMAX), torch.int32), ((Nloc, KMAX), torch.int32)]:
+        cnt = int(np.prod(shape))
+        views.append(rec[o:o + cnt].view(dt).view(shape))
+        o += cnt
+    gathered = [torch.empty_like(rec) for _ in range(world)] if (world > 1 and rank == 0) else None
+    titers = torch.zeros(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(count_iters=False):
+        if count_iters:
+            titers.zero_()
+        solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
+                     refill_threshold=a.refill, total_iters=titers if count_iters else None)
+        solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
+        if world > 1:
+            dist.gather(rec, gathered, dst=0)
+
+    for _ in range(max(a.warmup, 3)):
+        step()
+    step(count_iters=True)
+    torch.cuda.synchronize()
+    iters_local = int(titers.item())
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+           torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    l0 = solver.launch_count()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for i in range(a.steps):
+            flush.zero_()
+            e0, e1, e2 = ev[i]
+            e0.record(stream)
+            solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
+                         refill_threshold=a.refill)
+            e1.record(stream)
+            solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
+            if world > 1:
+                dist.gather(rec, gathered, dst=0)
+            e2.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches = solver.launch_count() - l0
+    t_step = [e0.elapsed_time(e2) for e0, e1, e2 in ev]
+    t_solve = [e0.elapsed_time(e1) for e0, e1, e2 in ev]
+    tot_ms = float(sum(t_step))
+    stats = torch.tensor([tot_ms, float(iters_local), float(sum(t_solve))], dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = stats[[0, 2]].clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        itsum = stats[1:2].clone()
+        dist.all_reduce(itsum, op=dist.ReduceOp.SUM)
+        tot_ms, solve_ms, iters_all = float(tmax[0]), float(tmax[1]), float(itsum[0])
+    else:
+        solve_ms, iters_all = float(stats[2]), float(stats[1])
+
+    # end to end through the C ABI on host buffers (pinned), per step
+    e2e = None
+    if not a.no_e2e:
+        ent_p = torch.from_numpy(ent_h).pin_memory()
+        st_p = torch.from_numpy(st_h).pin_memory()
+        outs = {"count": torch.empty(Nloc, dtype=torch.int32).pin_memory(),
+                "lambda": torch.empty((Nloc, KMAX), dtype=torch.float32).pin_memory(),
+                "x": torch.empty((Nloc, KMAX, n), dtype=torch.float32).pin_memory(),
+                "mult": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory(),
+                "rep": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()}
+        chunk = max(4096, Nloc // 8)
+        solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
+                        chunk_tensors=chunk, out=outs)
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(a.steps):
+            solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
+                            chunk_tensors=chunk, out=outs)
+        e2e_s = time.perf_counter() - t0
+        e2e_t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        e2e_s = float(e2e_t[0])
+        h2d = ent_h.nbytes + st_h.nbytes
+        d2h = sum(int(v.numel() * v.element_size()) for v in outs.values())
+        F = solver.paper_flops_per_iter
+        e2e = {"value": F * iters_all * a.steps / e2e_s / 1e9, "unit": "GFLOP/s", "h2d_bytes_per_step": h2d * world,
+               "d2h_bytes_per_step": d2h * world, "ms_per_step": 1e3 * e2e_s / a.steps,
+               "voxel_solves_per_s": Nloc * world * a.steps / e2e_s, "chunk_tensors": chunk}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    F = solver.paper_flops_per_iter
+    Fx = solver.exec_flops_per_iter
+    T = tot_ms / 1e3
+    value = F * iters_all * a.steps / T / 1e9
+    vps = Nloc * world * a.steps / T
+    pk = peaks()
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    fmax = pk.get("sm_max_mhz") or clk.max_mhz or 1965.0
+    peak_tflops = sms * 128 * 2 * fmax * 1e6 / 1e12
+    achieved = Fx * iters_local * a.steps / (solve_ms / 1e3) / 1e12     # rank-local solve kernel
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tf):
+        with open(tf) as fh:
+            traffic = json.load(fh).get(a.config)
+    cpu = None
+    if world == 1 and not a.no_cpu:
+        nv = a.cpu_voxels or (16384 if (m, n) == (4, 3) else 512)
+        r = cpu_oracle(cfg, min(nv, Nloc))
+        cpu = {"value": r["gflops"], "unit": "GFLOP/s", "cores": r["cores"], "kind": "oracle",
+               "sample": f"first {r['voxels']} of {Nloc} tensors x {S} starts (same workload), FP64 full-tensor "
+                         f"numpy oracle, {r['cores']} processes, {r['seconds']:.1f} s",
+               "voxel_solves_per_s": r["voxel_solves_per_s"]}
+    line = {
+        "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+        "ms_per_step": tot_ms / a.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "f32", "data": "synthetic",
+        "config": {"workload": a.config, "m": m, "n": n, "tensors_per_gpu": Nloc, "tensors_total": Nloc * world,
+                   "starts": S, "alpha": cfg["alpha"], "tol": cfg["tol"], "maxit": cfg["maxit"],
+                   "dedup": {"lam_tol": LAM_TOL, "ang_tol": ANG_TOL, "kmax": KMAX},
+                   "flop_count": "paper-style F_paper(m,n) x sum(iters), reading R12",
+                   "l2": "flushed between timed steps (512 MiB write outside the events)",
+                   "parallelism": f"tensor-range shards x{world}" + (" + NCCL gather of dedup records" if world > 1 else "")},
+        "voxel_solves_per_s": vps,
+        "start_solves_per_s": vps * S,
+        "mean_iters": iters_all / (Nloc * world * S),
+        "ms_solve_per_step": solve_ms / a.steps,
+        "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tflops, "unit": "TFLOP/s",
+                     "frac": achieved / peak_tflops, "traffic": traffic,
+                     "kernel": f"sshopm_solve_kernel<{m},{n}>",
+                     "peak_basis": f"{sms} SM x 128 FP32 lanes x 2 x {fmax:.0f} MHz (sm_max_mhz)",
+                     "flops_per_update": Fx},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+        "context": {"paper_gpu": "318 GFLOP/s paper-style (31% of 1030), Tesla C2050, 1024 tensors (P:L5, P:L350)"},
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,166 @@
+/*
+ * sshopm.h — C ABI of libsshopm.so: batched SS-HOPM (shifted symmetric
+ * higher-order power method) over many small symmetric tensors on B200.
+ *
+ * Paper: Ballard, Kolda, Plantenga, "Efficiently Computing Tensor Eigenvalues
+ * on a GPU", IPDPS-W 2011.  Citations "P:L<n>" are lines of that paper's text
+ * (reference/PAPER.md); "R<k>" are the readings listed in DESIGN.md.
+ *
+ * Conventions shared by every entry point
+ * ---------------------------------------
+ * - Every call returns an int status (SSHOPM_OK = 0 or an error code below)
+ *   and never aborts the process.  Argument checks are synchronous.
+ * - Pointers named d_* are DEVICE pointers owned by the caller; pointers named
+ *   h_* are HOST pointers owned by the caller.  The library never frees or
+ *   retains caller memory beyond the call (asynchronous kernels read/write it
+ *   until the stream reaches that point).
+ * - Floating point data are IEEE float32, integer data int32 / uint8, all
+ *   row-major and contiguous, no padding.
+ * - Device work is enqueued asynchronously on `stream` (a cudaStream_t passed
+ *   as void*; NULL = legacy default stream).  Launch errors are returned as
+ *   SSHOPM_ECUDA; errors raised while kernels run surface at the caller's
+ *   next synchronisation (documented CUDA behaviour).
+ * - A handle is immutable after sshopm_create, so concurrent calls on
+ *   different streams are safe.  N = 0 is a no-op returning SSHOPM_OK.
+ *
+ * Storage format of one tensor (Table I)
+ * ---------------------------------------------------------------------
+ * A symmetric A in R^[m,n] (Definition 1) is stored as its
+ * U = C(m+n-1, m) unique values (Property 1), one per index class,
+ * classes in the paper's lexicographic order of index representations
+ * (nondecreasing tensor indices).  entries[t][c] = a_{i_1..i_m} for
+ * class c of tensor t (reading R8: entry values, not polynomial coefficients).
+ */
+#ifndef SSHOPM_H
+#define SSHOPM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct sshopm_ctx* sshopm_t;
+
+enum {
+  SSHOPM_OK = 0,
+  SSHOPM_EINVAL = 1,       /* bad argument (null pointer with N > 0, m < 2, n < 1, S < 1, maxit < 0, NaN alpha/tol, ...) */
+  SSHOPM_EUNSUPPORTED = 2, /* (m, n) or S outside what this build was compiled for */
+  SSHOPM_ECUDA = 3,        /* CUDA runtime error at launch / copy (see sshopm_last_cuda_error) */
+  SSHOPM_ENOMEM = 4        /* host or device allocation failed */
+};
+
+/* Create a solver for tensors of order m and dimension n.
+ * Enumerates the index classes and coefficients (Sec. III) and selects the
+ * kernel specialised for (m, n) at compile time (Sec. V-D loop unrolling,
+ * P:L327-331).  Holds host state only; allocates no device memory.
+ * Errors: EINVAL (m < 2, n < 1, out == NULL), EUNSUPPORTED ((m, n) not built). */
+int sshopm_create(int m, int n, sshopm_t* out);
+
+/* Destroy a handle.  NULL is accepted (no-op). */
+int sshopm_destroy(sshopm_t h);
+
+/* U = C(m+n-1, m), the number of unique entries per tensor (Property 1). */
+int sshopm_num_unique(sshopm_t h, int* U);
+
+/* Write the U index representations, 0-based, lexicographic order,
+ * into host array h_idx[U][m].  For tests and documentation. */
+int sshopm_class_index(sshopm_t h, int32_t* h_idx);
+
+/* Flop counts per SS-HOPM iteration of one (tensor, start) lane:
+ *   *paper    = (m+2) U + (m+1) T1 + 5 n   (reading R12 of the paper's counting,
+ *               Eq. 4 + Eq. 6 + shift/normalise; T1 = n C(m+n-2, m-1); parity unpinned)
+ *   *executed = FP32 flops of this library's evaluation (FMA = 2 flops) —
+ *               the algorithmic count used for the ALU roofline.
+ * Either pointer may be NULL. */
+int sshopm_flops_per_iter(sshopm_t h, int64_t* paper, int64_t* executed);
+
+/* Batched SS-HOPM (Fig. 1; problem statement P:L305-307).
+ * For every tensor t < N and start s < S, runs SS-HOPM from x_0 = starts[s] /
+ * ||starts[s]|| (normalised on the device in FP32, reading R7):
+ *     lam_0 = A x_0^m; repeat  xhat = +-(A x_k^{m-1} + alpha x_k)  ("+" iff alpha >= 0, R5),
+ *                              x_{k+1} = xhat / ||xhat||, lam_{k+1} = A x_{k+1}^m
+ *     until |lam_{k+1} - lam_k| <= tol * max(1, |lam_{k+1}|) (converged, R2) or maxit updates.
+ * Outputs for lane (t, s) at index t*S + s:
+ *     d_out_lambda[N][S]   lam at the stopping update
+ *     d_out_x[N][S][n]     x at the stopping update (unit norm)
+ *     d_out_iters[N][S]    number of x-updates performed (Fig. 1 loop trips)
+ *     d_out_converged[N][S] 1 if the tolerance test fired, else 0
+ * Special cases: tol < 0 -> fixed-K mode (exactly maxit updates, converged = 0);
+ * maxit = 0 -> (lam_0, x_0), iters 0; a zero start or ||xhat|| = 0 stops the
+ * lane with converged = 0 and the last (lam, x) (R6).
+ * Inputs: d_entries[N][U], d_starts[S][n] (shared by all tensors).
+ * Errors: EINVAL (null pointers with N > 0, S < 1, maxit < 0, NaN alpha or tol),
+ *         ECUDA. */
+int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                 float alpha, float tol, int maxit,
+                 float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                 void* stream);
+
+/* Tuning / instrumentation knobs for sshopm_solve_ex (0 = library default). */
+typedef struct {
+  int refill_threshold;            /* lanes that must be idle before a warp refills (1..32); default per (m, n) */
+  int ctas_per_sm;                 /* persistent CTAs per SM; default = max occupancy */
+  unsigned long long* d_total_iters; /* optional device counter: += sum of iters over all lanes (atomicAdd) */
+} sshopm_solve_opts;
+
+/* sshopm_solve with options (opts may be NULL). */
+int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                    float alpha, float tol, int maxit,
+                    float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                    const sshopm_solve_opts* opts, void* stream);
+
+/* Per-tensor eigenpair dedup (reading R16).
+ * For each tensor t: visit converged starts in start order; a start joins the
+ * first existing cluster whose representative r has
+ *     |lam_s - lam_r| <= lam_tol * max(1, |lam_r|)  and  angle(x_s, x_r) <= ang_tol
+ * (sign-free for even m, R15; for odd m (lam, x) ~ (-lam, -x)), else it
+ * founds a new cluster.  Clusters are ordered by representative lam
+ * descending, ties by representative start ascending.
+ * Outputs: d_out_count[N] total clusters (may exceed kmax), and for the first
+ * kmax clusters d_out_lambda[N][kmax], d_out_x[N][kmax][n], d_out_mult[N][kmax]
+ * (members), d_out_rep[N][kmax] (representative start, -1 in empty slots;
+ * d_out_rep may be NULL).  Empty slots: lambda 0, x 0, mult 0.
+ * Inputs are sshopm_solve's outputs.  Errors: EINVAL (kmax < 1, negative
+ * tolerances, null pointers), EUNSUPPORTED (S > 1024), ECUDA. */
+int sshopm_dedup(sshopm_t h, int64_t N, int S,
+                 const float* d_lambda, const float* d_x, const uint8_t* d_converged,
+                 float lam_tol, float ang_tol, int kmax,
+                 int32_t* d_out_count, float* d_out_lambda, float* d_out_x, int32_t* d_out_mult,
+                 int32_t* d_out_rep, void* stream);
+
+/* Test hook: d_out_g[N][n] = A x^{m-1} (Eq. 6) and d_out_lam[N] = A x^m
+ * (Eq. 4 via Euler's identity x.(A x^{m-1})) for N (tensor, x) pairs, using
+ * exactly the solver's compiled evaluation.  d_x[N][n] is NOT normalised. */
+int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x,
+                 float* d_out_g, float* d_out_lam, void* stream);
+
+/* End-to-end call on HOST buffers: copies h_entries to the device in chunks,
+ * runs solve + dedup on each chunk, and copies the dedup records back, with
+ * copies and compute overlapped on internal streams.  Raw per-start outputs
+ * are returned only if the h_out_* raw pointers are non-NULL.  Blocks until
+ * done.  Host buffers should be pinned (cudaHostAlloc / registered) for full
+ * bandwidth.  Device memory is allocated and freed inside the call.
+ * Errors: as sshopm_solve and sshopm_dedup, plus ENOMEM. */
+int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, int S, const float* h_starts,
+                    float alpha, float tol, int maxit,
+                    float lam_tol, float ang_tol, int kmax,
+                    int32_t* h_out_count, float* h_out_lambda, float* h_out_x, int32_t* h_out_mult,
+                    int32_t* h_out_rep,
+                    float* h_raw_lambda, float* h_raw_x, int32_t* h_raw_iters, uint8_t* h_raw_converged,
+                    int64_t chunk_tensors, unsigned long long* h_total_iters);
+
+/* Number of kernels this handle has launched since creation (instrumentation). */
+int sshopm_launch_count(sshopm_t h, int64_t* count);
+
+/* Human-readable status string; also the text of the last CUDA error. */
+const char* sshopm_status_string(int code);
+const char* sshopm_last_cuda_error(void);
+
+/* Comma-separated list of (m,n) pairs compiled into this build, e.g. "2x3,4x3". */
+const char* sshopm_supported_shapes(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SSHOPM_H */

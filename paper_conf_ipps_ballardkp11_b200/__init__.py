@@ -1,0 +1,238 @@
+"""Batched SS-HOPM on B200 — thin Python binding over libsshopm.so (include/sshopm.h).
+
+Argument marshalling only: every step of the hot path runs in the CUDA
+kernels of the C-ABI library.  PyTorch provides device memory and streams.
+There is no CPU fallback: if the library is missing, every call raises.
+
+    import paper_conf_ipps_ballardkp11_b200 as sh
+    solver = sh.Solver(4, 3)
+    lam, x, iters, conv = solver.solve(entries, starts, alpha=0.0, tol=1e-6, maxit=100)
+    count, clam, cx, mult, rep = solver.dedup(lam, x, conv)
+"""
+import ctypes
+import os
+
+import numpy as np
+
+__all__ = ["Solver", "SSHOPMError", "lib", "supported_shapes", "library_path"]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+library_path = os.path.join(_HERE, "_lib", "libsshopm.so")
+_LIB = None
+
+OK, EINVAL, EUNSUPPORTED, ECUDA, ENOMEM = 0, 1, 2, 3, 4
+
+
+class SSHOPMError(RuntimeError):
+    def __init__(self, code, where):
+        msg = f"{where}: status {code} ({_status(code)})"
+        if code == ECUDA:
+            msg += ": " + lib().sshopm_last_cuda_error().decode()
+        super().__init__(msg)
+        self.code = code
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
+                ("d_total_iters", ctypes.c_void_p)]
+
+
+def lib():
+    """Load libsshopm.so (built by __graft_entry__.build()); raises if absent."""
+    global _LIB
+    if _LIB is not None:
+        return _LIB
+    if not os.path.exists(library_path):
+        raise RuntimeError(f"{library_path} is not built; run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = ctypes.CDLL(library_path)
+    P, I, I64, F = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_float
+    sig = {
+        "sshopm_create": (I, [I, I, ctypes.POINTER(P)]),
+        "sshopm_destroy": (I, [P]),
+        "sshopm_num_unique": (I, [P, ctypes.POINTER(I)]),
+        "sshopm_class_index": (I, [P, P]),
+        "sshopm_flops_per_iter": (I, [P, ctypes.POINTER(I64), ctypes.POINTER(I64)]),
+        "sshopm_solve": (I, [P, I64, P, I, P, F, F, I, P, P, P, P, P]),
+        "sshopm_solve_ex": (I, [P, I64, P, I, P, F, F, I, P, P, P, P, ctypes.POINTER(_Opts), P]),
+        "sshopm_dedup": (I, [P, I64, I, P, P, P, F, F, I, P, P, P, P, P, P]),
+        "sshopm_apply": (I, [P, I64, P, P, P, P, P]),
+        "sshopm_run_host": (I, [P, I64, P, I, P, F, F, I, F, F, I, P, P, P, P, P, P, P, P, P, I64, P]),
+        "sshopm_launch_count": (I, [P, ctypes.POINTER(I64)]),
+        "sshopm_status_string": (ctypes.c_char_p, [I]),
+        "sshopm_last_cuda_error": (ctypes.c_char_p, []),
+        "sshopm_supported_shapes": (ctypes.c_char_p, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _LIB = L
+    return L
+
+
+def _status(code):
+    return lib().sshopm_status_string(code).decode()
+
+
+def _check(code, where):
+    if code != OK:
+        raise SSHOPMError(code, where)
+
+
+def supported_shapes():
+    """[(m, n), ...] compiled into the library."""
+    s = lib().sshopm_supported_shapes().decode()
+    return [tuple(int(t) for t in p.split("x")) for p in s.split(",") if p]
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _dev(t, dtype, shape, name):
+    torch = _torch()
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA torch.Tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name} must have shape {tuple(shape)}, got {tuple(t.shape)}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream):
+    torch = _torch()
+    s = torch.cuda.current_stream() if stream is None else stream
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+class Solver:
+    """Handle for tensors of order m, dimension n (sshopm_create)."""
+
+    def __init__(self, m, n):
+        h = ctypes.c_void_p()
+        _check(lib().sshopm_create(int(m), int(n), ctypes.byref(h)), f"sshopm_create({m},{n})")
+        self._h = h
+        self.m, self.n = int(m), int(n)
+        u = ctypes.c_int()
+        _check(lib().sshopm_num_unique(h, ctypes.byref(u)), "sshopm_num_unique")
+        self.U = u.value
+        pf, ef = ctypes.c_int64(), ctypes.c_int64()
+        _check(lib().sshopm_flops_per_iter(h, ctypes.byref(pf), ctypes.byref(ef)), "sshopm_flops_per_iter")
+        self.paper_flops_per_iter = pf.value
+        self.exec_flops_per_iter = ef.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().sshopm_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def class_index(self):
+        out = np.zeros((self.U, self.m), dtype=np.int32)
+        _check(lib().sshopm_class_index(self._h, out.ctypes.data_as(ctypes.c_void_p)), "sshopm_class_index")
+        return out
+
+    def launch_count(self):
+        c = ctypes.c_int64()
+        _check(lib().sshopm_launch_count(self._h, ctypes.byref(c)), "sshopm_launch_count")
+        return c.value
+
+    def solve(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, out=None, refill_threshold=0,
+              ctas_per_sm=0, total_iters=None, stream=None):
+        """entries [N, U] f32, starts [S, n] f32 (CUDA) -> (lam [N,S], x [N,S,n], iters [N,S] i32, conv [N,S] u8)."""
+        torch = _torch()
+        N, S = int(entries.shape[0]), int(starts.shape[0])
+        pe = _dev(entries, torch.float32, (N, self.U), "entries")
+        ps = _dev(starts, torch.float32, (S, self.n), "starts")
+        dev = entries.device
+        if out is None:
+            out = (torch.empty((N, S), dtype=torch.float32, device=dev),
+                   torch.empty((N, S, self.n), dtype=torch.float32, device=dev),
+                   torch.empty((N, S), dtype=torch.int32, device=dev),
+                   torch.empty((N, S), dtype=torch.uint8, device=dev))
+        lam, x, it, cv = out
+        args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
+                _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
+        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None)
+        if total_iters is not None:
+            if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:
+                raise TypeError("total_iters must be a 1-element int64 CUDA tensor")
+            opts.d_total_iters = total_iters.data_ptr()
+        _check(lib().sshopm_solve_ex(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit), *args,
+                                     ctypes.byref(opts), _stream(stream)), "sshopm_solve")
+        return out
+
+    def dedup(self, lam, x, conv, lam_tol=1e-2, ang_tol=0.05, kmax=8, out=None, stream=None):
+        """-> (count [N] i32, lam [N,kmax], x [N,kmax,n], mult [N,kmax] i32, rep [N,kmax] i32)."""
+        torch = _torch()
+        N, S = int(lam.shape[0]), int(lam.shape[1])
+        pl = _dev(lam, torch.float32, (N, S), "lambda")
+        px = _dev(x, torch.float32, (N, S, self.n), "x")
+        pc = _dev(conv, torch.uint8, (N, S), "converged")
+        dev = lam.device
+        if out is None:
+            out = (torch.empty((N,), dtype=torch.int32, device=dev),
+                   torch.empty((N, kmax), dtype=torch.float32, device=dev),
+                   torch.empty((N, kmax, self.n), dtype=torch.float32, device=dev),
+                   torch.empty((N, kmax), dtype=torch.int32, device=dev),
+                   torch.empty((N, kmax), dtype=torch.int32, device=dev))
+        c, ol, ox, om, orp = out
+        _check(lib().sshopm_dedup(self._h, N, S, pl, px, pc, float(lam_tol), float(ang_tol), int(kmax),
+                                  _dev(c, torch.int32, (N,), "out_count"),
+                                  _dev(ol, torch.float32, (N, kmax), "out_lambda"),
+                                  _dev(ox, torch.float32, (N, kmax, self.n), "out_x"),
+                                  _dev(om, torch.int32, (N, kmax), "out_mult"),
+                                  _dev(orp, torch.int32, (N, kmax), "out_rep"), _stream(stream)), "sshopm_dedup")
+        return out
+
+    def apply(self, entries, x, stream=None):
+        """Test hook: (A x^{m-1} [N, n], A x^m [N]) with the solver's compiled evaluation."""
+        torch = _torch()
+        N = int(entries.shape[0])
+        pe = _dev(entries, torch.float32, (N, self.U), "entries")
+        px = _dev(x, torch.float32, (N, self.n), "x")
+        g = torch.empty((N, self.n), dtype=torch.float32, device=entries.device)
+        lam = torch.empty((N,), dtype=torch.float32, device=entries.device)
+        _check(lib().sshopm_apply(self._h, N, pe, px, ctypes.c_void_p(g.data_ptr()), ctypes.c_void_p(lam.data_ptr()),
+                                  _stream(stream)), "sshopm_apply")
+        return g, lam
+
+    def run_host(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, lam_tol=1e-2, ang_tol=0.05, kmax=8,
+                 raw=False, chunk_tensors=0, out=None):
+        """End-to-end on HOST arrays (numpy or pinned CPU torch tensors); returns a dict of host arrays."""
+        def ptr(a):
+            if hasattr(a, "data_ptr"):
+                if not a.is_contiguous():
+                    raise ValueError("host tensors must be contiguous")
+                return ctypes.c_void_p(a.data_ptr())
+            if not a.flags["C_CONTIGUOUS"]:
+                raise ValueError("host arrays must be C-contiguous")
+            return ctypes.c_void_p(a.ctypes.data)
+
+        N, S = int(entries.shape[0]), int(starts.shape[0])
+        if tuple(entries.shape) != (N, self.U) or tuple(starts.shape) != (S, self.n):
+            raise ValueError("entries must be [N, U] and starts [S, n]")
+        if out is None:
+            out = {"count": np.empty(N, np.int32), "lambda": np.empty((N, kmax), np.float32),
+                   "x": np.empty((N, kmax, self.n), np.float32), "mult": np.empty((N, kmax), np.int32),
+                   "rep": np.empty((N, kmax), np.int32)}
+            if raw:
+                out.update({"raw_lambda": np.empty((N, S), np.float32), "raw_x": np.empty((N, S, self.n), np.float32),
+                            "raw_iters": np.empty((N, S), np.int32), "raw_converged": np.empty((N, S), np.uint8)})
+        rawp = [ptr(out[k]) if raw else None for k in ("raw_lambda", "raw_x", "raw_iters", "raw_converged")]
+        tot = ctypes.c_ulonglong(0)
+        _check(lib().sshopm_run_host(self._h, N, ptr(entries), S, ptr(starts), float(alpha), float(tol), int(maxit),
+                                     float(lam_tol), float(ang_tol), int(kmax), ptr(out["count"]), ptr(out["lambda"]),
+                                     ptr(out["x"]), ptr(out["mult"]), ptr(out["rep"]), *rawp, int(chunk_tensors),
+                                     ctypes.byref(tot)), "sshopm_run_host")
+        out["total_iters"] = tot.value
+        return out

@@ -1,0 +1,266 @@
+// sshopm_api.cu — the C ABI of libsshopm.so (declared in include/sshopm.h).
+//
+// Argument validation, dispatch over the compiled (m, n) instances
+// (shapes.def), launch sizing from the device's SM count and the kernel's
+// occupancy, and the dedup kernels.  No device memory is allocated here
+// except inside sshopm_run_host (host_pipeline.cu).
+#include <atomic>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "launchers.h"
+#include "sshopm.h"
+#include "sshopm_dedup.cuh"
+#include "api_internal.h"
+
+namespace sshopm {
+#define SHAPE(mm, nn) const Launchers* get_launchers_##mm##_##nn();
+#include "shapes.def"
+#undef SHAPE
+
+static const Launchers* find_launchers(int m, int n) {
+#define SHAPE(mm, nn) if (m == mm && n == nn) return get_launchers_##mm##_##nn();
+#include "shapes.def"
+#undef SHAPE
+  return nullptr;
+}
+
+static thread_local char g_last_cuda_error[512] = "";
+
+int cuda_fail(cudaError_t e, const char* where) {
+  snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "%s: %s (%s)", where, cudaGetErrorName(e), cudaGetErrorString(e));
+  return SSHOPM_ECUDA;
+}
+
+FastDiv make_fastdiv(uint32_t d) {
+  FastDiv f;
+  f.d = d;
+  uint32_t s = 0;
+  while ((1ull << s) < d) ++s;
+  f.shift = s;
+  f.magic = (uint32_t)((((1ull << 32) * ((1ull << s) - d)) / d) + 1);
+  return f;
+}
+
+int device_sms() {
+  int dev = 0, sms = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return -1;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return -1;
+  return sms;
+}
+}  // namespace sshopm
+
+using namespace sshopm;
+
+extern "C" {
+
+const char* sshopm_status_string(int code) {
+  switch (code) {
+    case SSHOPM_OK: return "ok";
+    case SSHOPM_EINVAL: return "invalid argument";
+    case SSHOPM_EUNSUPPORTED: return "unsupported shape or size";
+    case SSHOPM_ECUDA: return "CUDA error (see sshopm_last_cuda_error)";
+    case SSHOPM_ENOMEM: return "out of memory";
+    default: return "unknown status";
+  }
+}
+
+const char* sshopm_last_cuda_error(void) { return g_last_cuda_error; }
+
+const char* sshopm_supported_shapes(void) {
+  static const char* s =
+#define SHAPE(mm, nn) #mm "x" #nn ","
+#include "shapes.def"
+#undef SHAPE
+      "";
+  return s;
+}
+
+int sshopm_create(int m, int n, sshopm_t* out) {
+  if (!out || m < 2 || n < 1) return SSHOPM_EINVAL;
+  *out = nullptr;
+  const Launchers* L = find_launchers(m, n);
+  if (!L) return SSHOPM_EUNSUPPORTED;
+  sshopm_ctx* h = new (std::nothrow) sshopm_ctx;
+  if (!h) return SSHOPM_ENOMEM;
+  h->L = L;
+  h->launches.store(0);
+  *out = h;
+  return SSHOPM_OK;
+}
+
+int sshopm_destroy(sshopm_t h) {
+  delete h;
+  return SSHOPM_OK;
+}
+
+int sshopm_num_unique(sshopm_t h, int* U) {
+  if (!h || !U) return SSHOPM_EINVAL;
+  *U = h->L->U;
+  return SSHOPM_OK;
+}
+
+int sshopm_class_index(sshopm_t h, int32_t* h_idx) {
+  if (!h || !h_idx) return SSHOPM_EINVAL;
+  h->L->class_index(h_idx);
+  return SSHOPM_OK;
+}
+
+int sshopm_flops_per_iter(sshopm_t h, int64_t* paper, int64_t* executed) {
+  if (!h) return SSHOPM_EINVAL;
+  if (paper) *paper = h->L->paper_flops;
+  if (executed) *executed = h->L->exec_flops;
+  return SSHOPM_OK;
+}
+
+int sshopm_launch_count(sshopm_t h, int64_t* count) {
+  if (!h || !count) return SSHOPM_EINVAL;
+  *count = h->launches.load();
+  return SSHOPM_OK;
+}
+
+int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                    float alpha, float tol, int maxit,
+                    float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                    const sshopm_solve_opts* opts, void* stream) {
+  if (!h || N < 0 || S < 1 || maxit < 0 || std::isnan(alpha) || std::isnan(tol)) return SSHOPM_EINVAL;
+  if (N == 0) return SSHOPM_OK;
+  if (!d_entries || !d_starts || !d_out_lambda || !d_out_x || !d_out_iters || !d_out_converged) return SSHOPM_EINVAL;
+  if (N > (1LL << 40) / S) return SSHOPM_EUNSUPPORTED;
+  const Launchers* L = h->L;
+  const int n = L->n;
+  const long long total = (long long)N * S;
+  const int sms = device_sms();
+  if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
+
+  const int smem = (S * n * 4 <= 64 * 1024) ? S * n * 4 : 0;
+  const bool neg = alpha < 0.f;
+  int bps = 0;
+  cudaError_t e = L->occupancy(neg, smem, &bps);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
+  if (bps < 1) bps = 1;
+  if (opts && opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
+  const long long warps_full = (long long)sms * bps * 8;
+  long long ipw = (total + warps_full - 1) / warps_full;
+  if (ipw < 64) ipw = 64;                       // keep lanes busy on small problems
+  if (ipw > (1LL << 30)) return SSHOPM_EUNSUPPORTED;
+  const long long warps = (total + ipw - 1) / ipw;
+  const long long grid = (warps + 7) / 8;
+
+  SolveParams p;
+  p.entries = d_entries;
+  p.starts = d_starts;
+  p.out_lambda = d_out_lambda;
+  p.out_x = d_out_x;
+  p.out_iters = d_out_iters;
+  p.out_conv = d_out_converged;
+  p.total_iters = opts ? opts->d_total_iters : nullptr;
+  p.total_items = total;
+  p.items_per_warp = ipw;
+  p.S = S;
+  p.divS = make_fastdiv((uint32_t)S);
+  p.alpha = alpha;
+  p.tol = tol;
+  p.maxit = maxit;
+  int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : L->default_refill;
+  p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
+  p.starts_in_smem = smem > 0 ? 1 : 0;
+  e = L->solve(p, neg, (int)grid, smem, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: launch");
+  h->launches.fetch_add(1);
+  return SSHOPM_OK;
+}
+
+int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                 float alpha, float tol, int maxit,
+                 float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                 void* stream) {
+  return sshopm_solve_ex(h, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
+                         d_out_converged, nullptr, stream);
+}
+
+int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x,
+                 float* d_out_g, float* d_out_lam, void* stream) {
+  if (!h || N < 0) return SSHOPM_EINVAL;
+  if (N == 0) return SSHOPM_OK;
+  if (!d_entries || !d_x || !d_out_g || !d_out_lam) return SSHOPM_EINVAL;
+  const int sms = device_sms();
+  if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_apply: no device");
+  long long grid = (N + 255) / 256;
+  if (grid > (long long)sms * 16) grid = (long long)sms * 16;
+  cudaError_t e = h->L->apply(N, d_entries, d_x, d_out_g, d_out_lam, (int)grid, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_apply: launch");
+  h->launches.fetch_add(1);
+  return SSHOPM_OK;
+}
+
+}  // extern "C"
+
+namespace sshopm {
+template <int NN, bool EVEN>
+static cudaError_t launch_dedup(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup_kernel<NN, EVEN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+  }
+  sshopm_dedup_kernel<NN, EVEN><<<grid, block, smem, st>>>(p);
+  return cudaGetLastError();
+}
+
+int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
+               float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
+               int32_t* d_rep, cudaStream_t st) {
+  if (S < 1 || kmax < 1 || !(lam_tol >= 0.f) || !(ang_tol >= 0.f) || N < 0) return SSHOPM_EINVAL;
+  if (N == 0) return SSHOPM_OK;
+  if (!d_lambda || !d_x || !d_conv || !d_count || !d_olam || !d_ox || !d_mult) return SSHOPM_EINVAL;
+  if (S > 1024) return SSHOPM_EUNSUPPORTED;
+  const int n = L->n;
+  const int sms = device_sms();
+  if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_dedup: no device");
+  const int per_warp = dedup_smem_words(S, n) * 4;
+  int wpb = (96 * 1024) / per_warp;
+  if (wpb > 8) wpb = 8;
+  if (wpb < 1) wpb = 1;
+  const int smem = wpb * per_warp;
+  long long grid = (N + wpb - 1) / wpb;
+  if (grid > (long long)sms * 16) grid = (long long)sms * 16;
+  DedupParams p;
+  p.lambda = d_lambda;
+  p.x = d_x;
+  p.conv = d_conv;
+  p.out_count = d_count;
+  p.out_lambda = d_olam;
+  p.out_x = d_ox;
+  p.out_mult = d_mult;
+  p.out_rep = d_rep;
+  p.n_tensors = N;
+  p.S = S;
+  p.kmax = kmax;
+  p.lam_tol = lam_tol;
+  p.cos_tol = ang_tol >= 3.14159265358979f ? -1.0f : cosf(ang_tol);
+  const bool even = (L->m % 2) == 0;
+  cudaError_t e = cudaErrorInvalidValue;
+  switch (n) {
+#define DD(NN) case NN: e = even ? launch_dedup<NN, true>(p, (int)grid, 32 * wpb, smem, st) : launch_dedup<NN, false>(p, (int)grid, 32 * wpb, smem, st); break;
+    DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
+#undef DD
+    default: return SSHOPM_EUNSUPPORTED;
+  }
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_dedup: launch");
+  return SSHOPM_OK;
+}
+}  // namespace sshopm
+
+extern "C" int sshopm_dedup(sshopm_t h, int64_t N, int S,
+                            const float* d_lambda, const float* d_x, const uint8_t* d_converged,
+                            float lam_tol, float ang_tol, int kmax,
+                            int32_t* d_out_count, float* d_out_lambda, float* d_out_x, int32_t* d_out_mult,
+                            int32_t* d_out_rep, void* stream) {
+  if (!h) return SSHOPM_EINVAL;
+  int r = dedup_impl(h->L, N, S, d_lambda, d_x, d_converged, lam_tol, ang_tol, kmax, d_out_count, d_out_lambda,
+                     d_out_x, d_out_mult, d_out_rep, (cudaStream_t)stream);
+  if (r == SSHOPM_OK && N > 0) h->launches.fetch_add(1);
+  return r;
+}

@@ -1,0 +1,232 @@
+"""GPU parity tests: CUDA path (through the C ABI) vs the FP64 oracle.
+
+Run on a B200 with ``pytest -m gpu``.  Inputs come from synthetic/ (seeded);
+expected values come only from oracle/.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_ipps_ballardkp11_b200 as sh  # noqa: E402
+import synthetic as syn  # noqa: E402
+from oracle import sshopm as O  # noqa: E402
+from oracle import dedup as D  # noqa: E402
+from tests import parity as PR  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def dev():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch.device("cuda:0")
+
+
+def _solve(dev, m, n, ent, st, alpha, tol, maxit, **kw):
+    s = sh.Solver(m, n)
+    out = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), alpha, tol, maxit, **kw)
+    torch.cuda.synchronize()
+    return tuple(t.cpu().numpy() for t in out)
+
+
+def _assert_parity(rep, max_sensitive=1e-3):
+    """P1-P3 with zero unexplained lanes; explained (precision-sensitive) lanes must stay rare."""
+    print({k: v for k, v in rep.items() if k != "details"})
+    assert rep["flag_unexplained"] == 0, rep
+    assert rep["lam_unexplained"] == 0, rep
+    assert rep.get("angle_unexplained", 0) == 0, rep
+    assert rep["sensitive_frac"] <= max_sensitive, rep
+
+
+# ---------------------------------------------------------------- apply (T2) --
+def _exact_inputs(m, n, count, seed):
+    amax = 5
+    xmax = 3 if m <= 4 else 1
+    return syn.gen_small_int(m, n, count, seed, amax), syn.gen_int_vectors(count, n, seed + 1, xmax)
+
+
+@pytest.mark.parametrize("m,n", [(2, 2), (2, 3), (2, 4), (3, 2), (3, 3), (3, 4), (4, 2), (4, 3), (4, 4), (4, 5),
+                                 (4, 6), (5, 3), (6, 2), (6, 3), (8, 3)])
+def test_apply_exact_on_integers(dev, m, n):
+    """Eq. 6 and Eq. 4 (Euler) in FP32 == FP64 full-tensor oracle, bit-exact on small integers."""
+    ent, x = _exact_inputs(m, n, 1000, m * 7 + n)
+    s = sh.Solver(m, n)
+    g, lam = s.apply(torch.from_numpy(ent).to(dev), torch.from_numpy(x).to(dev))
+    full = O.expand_full(ent, m, n)
+    g_ref = O.axm1(full, x.astype(np.float64))
+    lam_ref = O.axm(full, x.astype(np.float64))
+    assert np.abs(g_ref).max() < 2 ** 24 and np.abs(lam_ref).max() < 2 ** 24
+    assert np.array_equal(g.cpu().numpy().astype(np.float64), g_ref)
+    assert np.array_equal(lam.cpu().numpy().astype(np.float64), lam_ref)
+
+
+def test_apply_random_close(dev):
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 4096, 1)
+    x = O.normalise_starts(syn.gen_starts(4096, n, 3)).astype(np.float32)
+    g, lam = sh.Solver(m, n).apply(torch.from_numpy(ent).to(dev), torch.from_numpy(x).to(dev))
+    full = O.expand_full(ent, m, n)
+    assert np.allclose(g.cpu().numpy(), O.axm1(full, x.astype(np.float64)), atol=2e-6)
+    assert np.allclose(lam.cpu().numpy(), O.axm(full, x.astype(np.float64)), atol=2e-6)
+
+
+# ------------------------------------------------------------ solve parity --
+def test_parity_C1_full(dev):
+    """Config C1: all 1024 x 128 lanes, alpha = 0, tol 1e-6, maxit 100."""
+    c = syn.CONFIGS["C1"]
+    m, n = c["m"], c["n"]
+    ent = syn.gen_voxels(m, n, 0, c["N"], 0)
+    st = syn.gen_starts(c["S"], n, 0)
+    gpu = _solve(dev, m, n, ent, st, c["alpha"], c["tol"], c["maxit"])
+    rep = PR.solve_parity(ent, st, m, n, c["alpha"], c["tol"], c["maxit"], gpu)
+    _assert_parity(rep)
+    assert rep["gpu_converged"] > 0.99
+    assert np.allclose(np.linalg.norm(gpu[1], axis=2), 1.0, atol=1e-6)
+
+
+@pytest.mark.parametrize("m,n,V,alpha", [(4, 3, 256, 0.5), (4, 3, 128, -0.5), (6, 3, 128, 0.25), (8, 3, 24, 0.5),
+                                         (4, 6, 64, 0.0), (2, 3, 64, 1.0), (3, 3, 64, 1.0), (3, 2, 64, 0.5),
+                                         (4, 5, 32, 0.0), (5, 3, 32, 0.5), (6, 2, 64, 0.25), (4, 4, 64, 0.25)])
+def test_parity_shapes(dev, m, n, V, alpha):
+    """Other orders / dimensions / shifts.  Odd m uses unstructured U[-1,1] tensors and alpha < 0 seeks
+    minima below the concavity bound, so more lanes are precision-sensitive there (<= 5%)."""
+    ent = syn.gen_voxels(m, n, 12345, V, 2) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 2)
+    st = syn.gen_starts(128, n, 5)
+    gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 100)
+    stress = m % 2 == 1 or alpha < 0
+    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 100, gpu), 0.05 if stress else 1e-3)
+
+
+@pytest.mark.parametrize("alpha,K", [(0.0, 1), (0.0, 5), (0.0, 10), (0.5, 5), (0.5, 10)])
+def test_fixed_k(dev, alpha, K):
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 256, 0)
+    st = syn.gen_starts(128, n, 0)
+    lam, x, it, cv = _solve(dev, m, n, ent, st, alpha, -1.0, K)
+    assert (it == K).all() and not cv.any()
+    r = PR.fixed_k_parity(ent, st, m, n, alpha, K, lam)
+    print(r)
+    assert r["unexplained"] == 0, r
+
+
+def test_special_cases(dev):
+    """maxit = 0 -> (lam_0, x_0); zero start -> 0; odd S, N not a multiple of anything."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 37, 0)
+    st = syn.gen_starts(13, n, 0)
+    st[4] = 0.0
+    lam, x, it, cv = _solve(dev, m, n, ent, st, 0.0, 1e-6, 0)
+    assert (it == 0).all() and not cv.any()
+    x0 = O.normalise_starts(st)
+    assert np.allclose(x, np.broadcast_to(x0, x.shape), atol=1e-7)
+    full = O.expand_full(ent, m, n)
+    lam0 = O.axm(np.repeat(full, 13, 0), np.tile(x0, (37, 1))).reshape(37, 13)
+    assert np.allclose(lam, lam0, atol=1e-5)
+    lam, x, it, cv = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
+    assert (lam[:, 4] == 0).all() and (x[:, 4] == 0).all() and (it[:, 4] == 0).all() and not cv[:, 4].any()
+    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, (lam, x, it, cv)))
+
+
+def test_invariance_across_launch_configs(dev):
+    """T4: per-lane arithmetic is order-fixed -> bitwise identical across refill thresholds / grid sizes."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 2048, 3)
+    st = syn.gen_starts(128, n, 0)
+    base = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
+    for kw in [dict(refill_threshold=1), dict(refill_threshold=32), dict(ctas_per_sm=1),
+               dict(refill_threshold=5, ctas_per_sm=2), {}]:
+        other = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, **kw)
+        for a, b in zip(base, other):
+            assert np.array_equal(a, b), kw
+
+
+def test_total_iters_counter(dev):
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 512, 0)
+    st = syn.gen_starts(128, n, 0)
+    ti = torch.zeros(1, dtype=torch.int64, device=dev)
+    lam, x, it, cv = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, total_iters=ti)
+    assert int(ti.item()) == int(it.sum())
+
+
+# ------------------------------------------------------------------ dedup --
+def test_dedup_kernel_matches_oracle_rule_on_same_lanes(dev):
+    """GPU dedup vs oracle dedup applied to the GPU's own per-lane results."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 1024, 0)
+    st = syn.gen_starts(128, n, 0)
+    s = sh.Solver(m, n)
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.0, 1e-6, 100)
+    for lt, at, kmax in [(1e-2, 0.05, 8), (1e-3, 0.01, 4), (1e-1, 0.5, 2)]:
+        cnt, cl, cx, mu, rp = (t.cpu().numpy() for t in s.dedup(lam, x, cv, lt, at, kmax))
+        oc, ol, ox, om, orp = D.dedup(lam.cpu().numpy(), x.cpu().numpy(), cv.cpu().numpy().astype(bool), m, lt, at, kmax)
+        assert np.array_equal(cnt, oc)
+        assert np.array_equal(rp, orp)
+        assert np.array_equal(mu, om)
+        assert np.array_equal(cl.astype(np.float64), ol)
+        assert np.array_equal(cx.astype(np.float64), ox)
+
+
+def test_dedup_end_to_end_vs_oracle(dev):
+    """solve + dedup on GPU vs oracle solve + oracle dedup: identical cluster structure."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 512, 4)
+    st = syn.gen_starts(128, n, 0)
+    s = sh.Solver(m, n)
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.0, 1e-6, 100)
+    cnt, cl, cx, mu, rp = (t.cpu().numpy() for t in s.dedup(lam, x, cv, 1e-2, 0.05, 8))
+    rl, rx, ri, rc = O.sshopm(ent, st, m, n, 0.0, 1e-6, 100)
+    oc, ol, ox, om, orp = D.dedup(rl, rx, rc, m, 1e-2, 0.05, 8)
+    flag_diff_vox = np.any(cv.cpu().numpy().astype(bool) != rc, axis=1)
+    same = ~flag_diff_vox
+    assert same.mean() > 0.98
+    assert np.array_equal(cnt[same], oc[same])
+    assert np.array_equal(rp[same], orp[same])
+    assert np.array_equal(mu[same], om[same])
+    filled = rp[same] >= 0
+    assert np.all(np.abs(cl[same][filled] - ol[same][filled]) <= 1e-4 * np.maximum(1, np.abs(ol[same][filled])))
+
+
+def test_dedup_odd_m(dev):
+    m, n = 3, 3
+    ent = syn.gen_uniform_tensors(m, n, 128, 1)
+    st = syn.gen_starts(128, n, 0)
+    s = sh.Solver(m, n)
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 1.0, 1e-6, 200)
+    cnt, cl, cx, mu, rp = (t.cpu().numpy() for t in s.dedup(lam, x, cv, 1e-2, 0.05, 8))
+    oc, ol, ox, om, orp = D.dedup(lam.cpu().numpy(), x.cpu().numpy(), cv.cpu().numpy().astype(bool), m, 1e-2, 0.05, 8)
+    assert np.array_equal(cnt, oc) and np.array_equal(rp, orp) and np.array_equal(mu, om)
+
+
+# --------------------------------------------------------------- host path --
+def test_run_host_matches_device_path(dev):
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 3000, 9)
+    st = syn.gen_starts(128, n, 0)
+    s = sh.Solver(m, n)
+    out = s.run_host(ent, st, 0.0, 1e-6, 100, 1e-2, 0.05, 8, raw=True, chunk_tensors=700)
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.0, 1e-6, 100)
+    cnt, cl, cx, mu, rp = s.dedup(lam, x, cv, 1e-2, 0.05, 8)
+    torch.cuda.synchronize()
+    assert np.array_equal(out["raw_lambda"], lam.cpu().numpy())
+    assert np.array_equal(out["raw_x"], x.cpu().numpy())
+    assert np.array_equal(out["raw_iters"], it.cpu().numpy())
+    assert np.array_equal(out["raw_converged"], cv.cpu().numpy())
+    assert np.array_equal(out["count"], cnt.cpu().numpy())
+    assert np.array_equal(out["rep"], rp.cpu().numpy())
+    assert np.array_equal(out["lambda"], cl.cpu().numpy())
+    assert out["total_iters"] == int(it.cpu().numpy().sum())
+
+
+def test_empty_and_tiny(dev):
+    m, n = 4, 3
+    s = sh.Solver(m, n)
+    e0 = torch.zeros((0, 15), device=dev)
+    st = torch.from_numpy(syn.gen_starts(8, 3, 0)).to(dev)
+    lam, x, it, cv = s.solve(e0, st)
+    assert lam.shape == (0, 8)
+    ent = syn.gen_voxels(m, n, 0, 1, 0)
+    st1 = syn.gen_starts(1, n, 0)
+    gpu = _solve(dev, m, n, ent, st1, 0.0, 1e-6, 100)
+    _assert_parity(PR.solve_parity(ent, st1, m, n, 0.0, 1e-6, 100, gpu))

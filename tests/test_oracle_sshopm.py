@@ -128,7 +128,7 @@ def test_kr_alpha0_not_monotone(golden_dir):
     tr = []
     O.sshopm_lanes(lambda idx: full[np.zeros(len(idx), int)], x0, 0.0, -1.0, 20, trace=tr)
     lam_hist = np.full((21, 64), np.nan)
-    for k, ids, ln in tr:
+    for k, ids, ln, _ in tr:
         lam_hist[k, ids] = ln
     dec = np.nanmin(np.diff(lam_hist[1:], axis=0), axis=0)
     assert (dec < -1e-6).sum() > 32
@@ -146,7 +146,7 @@ def test_monotone_above_convexity_bound(m, n):
         tr = []
         O.sshopm_lanes(lambda idx: full[np.zeros(len(idx), int)], x0, alpha, -1.0, 30, trace=tr)
         prev = lam0.copy()
-        for k, ids, ln in tr:
+        for k, ids, ln, _ in tr:
             assert np.all(ln >= prev[ids] - 1e-12 * np.maximum(1, np.abs(ln)))
             prev[ids] = ln
 
