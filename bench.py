@@ -295,7 +295,7 @@ def main():
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         e2e_s = float(e2e_t[0])
         h2d = ent_h.nbytes + st_h.nbytes
-        d2h = sum(int(v.numel() * v.element_size()) for v in outs.values())
+        d2h = sum(int(v.numel() * v.element_size()) for k, v in outs.items() if k != "total_iters")
         F = solver.paper_flops_per_iter
         e2e = {"value": F * iters_all * a.steps / e2e_s / 1e9, "unit": "GFLOP/s", "h2d_bytes_per_step": h2d * world,
                "d2h_bytes_per_step": d2h * world, "ms_per_step": 1e3 * e2e_s / a.steps,

@@ -34,6 +34,7 @@
 #ifndef SSHOPM_H
 #define SSHOPM_H
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -97,14 +98,23 @@ int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const flo
                  float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
                  void* stream);
 
-/* Tuning / instrumentation knobs for sshopm_solve_ex (0 = library default). */
+/* Device workspace needed by sshopm_solve_ex for N tensors (bytes): a 256-byte
+ * header (work counter) plus one 16-byte aligned packed coefficient row per
+ * tensor (precomputed coefficients).  sshopm_solve
+ * and sshopm_apply allocate it themselves (cudaMallocAsync on the stream). */
+int sshopm_workspace_size(sshopm_t h, int64_t N, size_t* bytes);
+
+/* Tuning / instrumentation knobs for sshopm_solve_ex (0 / NULL = library default). */
 typedef struct {
   int refill_threshold;            /* lanes that must be idle before a warp refills (1..32); default per (m, n) */
   int ctas_per_sm;                 /* persistent CTAs per SM; default = max occupancy */
   unsigned long long* d_total_iters; /* optional device counter: += sum of iters over all lanes (atomicAdd) */
+  void* d_workspace;               /* optional caller-owned device workspace, 256-byte aligned, >= sshopm_workspace_size */
+  size_t workspace_bytes;          /* its size; a too-small or misaligned workspace returns EINVAL */
 } sshopm_solve_opts;
 
-/* sshopm_solve with options (opts may be NULL). */
+/* sshopm_solve with options (opts may be NULL).  Launches two kernels on
+ * `stream`: the pack kernel (coefficient rows) and the solve kernel. */
 int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
                     float alpha, float tol, int maxit,
                     float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,

@@ -34,7 +34,8 @@ class SSHOPMError(RuntimeError):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
-                ("d_total_iters", ctypes.c_void_p)]
+                ("d_total_iters", ctypes.c_void_p), ("d_workspace", ctypes.c_void_p),
+                ("workspace_bytes", ctypes.c_size_t)]
 
 
 def lib():
@@ -58,6 +59,7 @@ def lib():
         "sshopm_apply": (I, [P, I64, P, P, P, P, P]),
         "sshopm_run_host": (I, [P, I64, P, I, P, F, F, I, F, F, I, P, P, P, P, P, P, P, P, P, I64, P]),
         "sshopm_launch_count": (I, [P, ctypes.POINTER(I64)]),
+        "sshopm_workspace_size": (I, [P, I64, ctypes.POINTER(ctypes.c_size_t)]),
         "sshopm_status_string": (ctypes.c_char_p, [I]),
         "sshopm_last_cuda_error": (ctypes.c_char_p, []),
         "sshopm_supported_shapes": (ctypes.c_char_p, []),
@@ -124,6 +126,7 @@ class Solver:
         _check(lib().sshopm_flops_per_iter(h, ctypes.byref(pf), ctypes.byref(ef)), "sshopm_flops_per_iter")
         self.paper_flops_per_iter = pf.value
         self.exec_flops_per_iter = ef.value
+        self._ws = None            # cached device workspace (torch uint8 tensor)
 
     def close(self):
         if getattr(self, "_h", None):
@@ -140,6 +143,21 @@ class Solver:
         out = np.zeros((self.U, self.m), dtype=np.int32)
         _check(lib().sshopm_class_index(self._h, out.ctypes.data_as(ctypes.c_void_p)), "sshopm_class_index")
         return out
+
+    def workspace_size(self, N):
+        b = ctypes.c_size_t()
+        _check(lib().sshopm_workspace_size(self._h, int(N), ctypes.byref(b)), "sshopm_workspace_size")
+        return b.value
+
+    def _workspace(self, N, device):
+        need = self.workspace_size(N)
+        ws = self._ws
+        if ws is None or ws.device != device or ws.numel() < need:
+            torch = _torch()
+            ws = torch.empty(need + 256, dtype=torch.uint8, device=device)
+            self._ws = ws
+        base = ws.data_ptr()
+        return ctypes.c_void_p((base + 255) // 256 * 256), need
 
     def launch_count(self):
         c = ctypes.c_int64()
@@ -162,7 +180,8 @@ class Solver:
         lam, x, it, cv = out
         args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
                 _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
-        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None)
+        wsp, wsb = self._workspace(N, dev) if N > 0 else (None, 0)
+        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb)
         if total_iters is not None:
             if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:
                 raise TypeError("total_iters must be a 1-element int64 CUDA tensor")

@@ -5,16 +5,30 @@
 #include <stdint.h>
 #include "launchers.h"
 
+namespace sshopm { struct HostCache; }
+
 struct sshopm_ctx {
   const sshopm::Launchers* L;
   std::atomic<long long> launches;
+  sshopm::HostCache* hc;     // run_host device buffers / streams (created lazily, guarded by its mutex)
 };
 
 namespace sshopm {
 int cuda_fail(cudaError_t e, const char* where);
 FastDiv make_fastdiv(uint32_t d);
 int device_sms();
+
+struct Workspace {
+  void* base = nullptr;
+  unsigned int* counter = nullptr;   // 256-byte header: chunk counter of the solve kernel
+  float4* packed = nullptr;          // [N][PW/4] packed coefficient rows
+  bool owned = false;
+};
+size_t workspace_bytes(const Launchers* L, int64_t N);
+int acquire_workspace(const Launchers* L, int64_t N, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws);
+int release_workspace(Workspace* ws, cudaStream_t st);
 int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
                float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
                int32_t* d_rep, cudaStream_t st);
+void free_host_cache(sshopm_ctx* h);
 }  // namespace sshopm

@@ -5,15 +5,19 @@
 // chunk, the solve/dedup kernels of another and the device->host copy of a
 // third overlap (copy engines and SMs work concurrently).  Only the per-tensor
 // dedup records (and optionally the raw per-start outputs) come back.
+//
+// Device buffers and streams are cached in the handle (HostCache) and reused
+// across calls — allocation, not transfer, would otherwise dominate; calls on
+// one handle serialise on the cache mutex.  sshopm_destroy frees the cache.
 #include <cstring>
-#include <vector>
+#include <mutex>
 
 #include "api_internal.h"
 #include "sshopm.h"
 
 using namespace sshopm;
 
-namespace {
+namespace sshopm {
 constexpr int kSlots = 3;
 
 struct Slot {
@@ -21,16 +25,47 @@ struct Slot {
   float *ent = nullptr, *lam = nullptr, *x = nullptr, *olam = nullptr, *ox = nullptr;
   int32_t *it = nullptr, *cnt = nullptr, *mult = nullptr, *rep = nullptr;
   uint8_t* cv = nullptr;
+  void* ws = nullptr;
+  size_t ws_bytes = 0;
 };
 
-void free_slot(Slot& s) {
-  if (s.st) cudaStreamSynchronize(s.st);
-  cudaFree(s.ent); cudaFree(s.lam); cudaFree(s.x); cudaFree(s.olam); cudaFree(s.ox);
-  cudaFree(s.it); cudaFree(s.cnt); cudaFree(s.mult); cudaFree(s.rep); cudaFree(s.cv);
-  if (s.st) cudaStreamDestroy(s.st);
-  s = Slot();
+struct HostCache {
+  std::mutex mu;
+  int device = -1;
+  long long chunk = 0;
+  int S = 0, kmax = 0;
+  Slot slots[kSlots];
+  float* d_starts = nullptr;
+  unsigned long long* d_total = nullptr;
+};
+
+static void free_slots(HostCache* c) {
+  for (int i = 0; i < kSlots; ++i) {
+    Slot& s = c->slots[i];
+    if (s.st) cudaStreamSynchronize(s.st);
+    cudaFree(s.ent); cudaFree(s.lam); cudaFree(s.x); cudaFree(s.olam); cudaFree(s.ox);
+    cudaFree(s.it); cudaFree(s.cnt); cudaFree(s.mult); cudaFree(s.rep); cudaFree(s.cv); cudaFree(s.ws);
+    if (s.st) cudaStreamDestroy(s.st);
+    s = Slot();
+  }
+  cudaFree(c->d_starts);
+  cudaFree(c->d_total);
+  c->d_starts = nullptr;
+  c->d_total = nullptr;
+  c->chunk = 0;
 }
-}  // namespace
+
+void free_host_cache(sshopm_ctx* h) {
+  if (!h->hc) return;
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (h->hc->device >= 0) cudaSetDevice(h->hc->device);
+  free_slots(h->hc);
+  if (cur >= 0) cudaSetDevice(cur);
+  delete h->hc;
+  h->hc = nullptr;
+}
+}  // namespace sshopm
 
 extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, int S, const float* h_starts,
                                float alpha, float tol, int maxit, float lam_tol, float ang_tol, int kmax,
@@ -47,39 +82,60 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   long long chunk = chunk_tensors > 0 ? chunk_tensors : 65536;
   if (chunk > N) chunk = N;
 
+  if (!h->hc) {
+    h->hc = new (std::nothrow) HostCache;
+    if (!h->hc) return SSHOPM_ENOMEM;
+  }
+  HostCache* c = h->hc;
+  std::lock_guard<std::mutex> lock(c->mu);
+  int dev = 0;
+  cudaGetDevice(&dev);
   int rc = SSHOPM_OK;
-  Slot slots[kSlots];
-  float* d_starts = nullptr;
-  unsigned long long* d_total = nullptr;
   cudaError_t e = cudaSuccess;
 #define CK(call, where) do { e = (call); if (e != cudaSuccess) { rc = (e == cudaErrorMemoryAllocation) ? SSHOPM_ENOMEM : cuda_fail(e, where); goto done; } } while (0)
-  CK(cudaMalloc(&d_starts, sizeof(float) * S * n), "run_host: malloc");
-  CK(cudaMalloc(&d_total, sizeof(unsigned long long)), "run_host: malloc");
-  for (int i = 0; i < kSlots && i * chunk < N; ++i) {
-    Slot& s = slots[i];
-    CK(cudaStreamCreateWithFlags(&s.st, cudaStreamNonBlocking), "run_host: stream");
-    CK(cudaMalloc(&s.ent, sizeof(float) * chunk * U), "run_host: malloc");
-    CK(cudaMalloc(&s.lam, sizeof(float) * chunk * S), "run_host: malloc");
-    CK(cudaMalloc(&s.x, sizeof(float) * chunk * S * n), "run_host: malloc");
-    CK(cudaMalloc(&s.it, sizeof(int32_t) * chunk * S), "run_host: malloc");
-    CK(cudaMalloc(&s.cv, chunk * S), "run_host: malloc");
-    CK(cudaMalloc(&s.cnt, sizeof(int32_t) * chunk), "run_host: malloc");
-    CK(cudaMalloc(&s.olam, sizeof(float) * chunk * kmax), "run_host: malloc");
-    CK(cudaMalloc(&s.ox, sizeof(float) * chunk * kmax * n), "run_host: malloc");
-    CK(cudaMalloc(&s.mult, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
-    CK(cudaMalloc(&s.rep, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
+  if (c->device != dev || c->chunk < chunk || c->S != S || c->kmax < kmax) {
+    if (c->device >= 0) {
+      int cur = dev;
+      cudaSetDevice(c->device);
+      free_slots(c);
+      cudaSetDevice(cur);
+    }
+    c->device = dev;
+    c->S = S;
+    c->kmax = kmax;
+    CK(cudaMalloc(&c->d_starts, sizeof(float) * S * n), "run_host: malloc");
+    CK(cudaMalloc(&c->d_total, sizeof(unsigned long long)), "run_host: malloc");
+    for (int i = 0; i < kSlots; ++i) {
+      Slot& s = c->slots[i];
+      CK(cudaStreamCreateWithFlags(&s.st, cudaStreamNonBlocking), "run_host: stream");
+      CK(cudaMalloc(&s.ent, sizeof(float) * chunk * U), "run_host: malloc");
+      CK(cudaMalloc(&s.lam, sizeof(float) * chunk * S), "run_host: malloc");
+      CK(cudaMalloc(&s.x, sizeof(float) * chunk * S * n), "run_host: malloc");
+      CK(cudaMalloc(&s.it, sizeof(int32_t) * chunk * S), "run_host: malloc");
+      CK(cudaMalloc(&s.cv, chunk * S), "run_host: malloc");
+      CK(cudaMalloc(&s.cnt, sizeof(int32_t) * chunk), "run_host: malloc");
+      CK(cudaMalloc(&s.olam, sizeof(float) * chunk * kmax), "run_host: malloc");
+      CK(cudaMalloc(&s.ox, sizeof(float) * chunk * kmax * n), "run_host: malloc");
+      CK(cudaMalloc(&s.mult, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
+      CK(cudaMalloc(&s.rep, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
+      s.ws_bytes = workspace_bytes(h->L, chunk);
+      CK(cudaMalloc(&s.ws, s.ws_bytes), "run_host: malloc");
+    }
+    c->chunk = chunk;
   }
-  CK(cudaMemcpyAsync(d_starts, h_starts, sizeof(float) * S * n, cudaMemcpyHostToDevice, slots[0].st), "run_host: H2D");
-  CK(cudaMemsetAsync(d_total, 0, sizeof(unsigned long long), slots[0].st), "run_host: memset");
-  CK(cudaStreamSynchronize(slots[0].st), "run_host: sync");
+  CK(cudaMemcpyAsync(c->d_starts, h_starts, sizeof(float) * S * n, cudaMemcpyHostToDevice, c->slots[0].st), "run_host: H2D");
+  CK(cudaMemsetAsync(c->d_total, 0, sizeof(unsigned long long), c->slots[0].st), "run_host: memset");
+  CK(cudaStreamSynchronize(c->slots[0].st), "run_host: sync");
   for (long long c0 = 0, ci = 0; c0 < N; c0 += chunk, ++ci) {
-    Slot& s = slots[ci % kSlots];
+    Slot& s = c->slots[ci % kSlots];
     const long long cn = (N - c0 < chunk) ? (N - c0) : chunk;
     CK(cudaMemcpyAsync(s.ent, h_entries + c0 * U, sizeof(float) * cn * U, cudaMemcpyHostToDevice, s.st), "run_host: H2D");
     sshopm_solve_opts o;
     memset(&o, 0, sizeof(o));
-    o.d_total_iters = d_total;
-    rc = sshopm_solve_ex(h, cn, s.ent, S, d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, &o, s.st);
+    o.d_total_iters = c->d_total;
+    o.d_workspace = s.ws;
+    o.workspace_bytes = s.ws_bytes;
+    rc = sshopm_solve_ex(h, cn, s.ent, S, c->d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, &o, s.st);
     if (rc != SSHOPM_OK) goto done;
     rc = dedup_impl(h->L, cn, S, s.lam, s.x, s.cv, lam_tol, ang_tol, kmax, s.cnt, s.olam, s.ox, s.mult, s.rep, s.st);
     if (rc != SSHOPM_OK) goto done;
@@ -98,12 +154,15 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     }
   }
   for (int i = 0; i < kSlots; ++i)
-    if (slots[i].st) CK(cudaStreamSynchronize(slots[i].st), "run_host: sync");
-  if (h_total_iters) CK(cudaMemcpy(h_total_iters, d_total, sizeof(unsigned long long), cudaMemcpyDeviceToHost), "run_host: D2H");
+    if (c->slots[i].st) CK(cudaStreamSynchronize(c->slots[i].st), "run_host: sync");
+  if (h_total_iters) CK(cudaMemcpy(h_total_iters, c->d_total, sizeof(unsigned long long), cudaMemcpyDeviceToHost), "run_host: D2H");
 #undef CK
 done:
-  for (int i = 0; i < kSlots; ++i) free_slot(slots[i]);
-  cudaFree(d_starts);
-  cudaFree(d_total);
+  if (rc != SSHOPM_OK) {
+    for (int i = 0; i < kSlots; ++i)
+      if (c->slots[i].st) cudaStreamSynchronize(c->slots[i].st);
+    free_slots(c);
+    c->device = -1;
+  }
   return rc;
 }

@@ -44,6 +44,35 @@ FastDiv make_fastdiv(uint32_t d) {
   return f;
 }
 
+size_t workspace_bytes(const Launchers* L, int64_t N) { return 256 + (size_t)N * (size_t)L->PW * 4; }
+
+int acquire_workspace(const Launchers* L, int64_t N, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws) {
+  const size_t need = workspace_bytes(L, N);
+  ws->owned = false;
+  void* base = user;
+  if (!user || user_bytes < need || ((uintptr_t)user & 255)) {
+    if (user && user_bytes < need) return SSHOPM_EINVAL;
+    if (user && ((uintptr_t)user & 255)) return SSHOPM_EINVAL;
+    cudaError_t e = cudaMallocAsync(&base, need, st);
+    if (e == cudaErrorMemoryAllocation) return SSHOPM_ENOMEM;
+    if (e != cudaSuccess) return cuda_fail(e, "workspace: cudaMallocAsync");
+    ws->owned = true;
+  }
+  ws->base = base;
+  ws->counter = reinterpret_cast<unsigned int*>(base);
+  ws->packed = reinterpret_cast<float4*>(reinterpret_cast<char*>(base) + 256);
+  return SSHOPM_OK;
+}
+
+int release_workspace(Workspace* ws, cudaStream_t st) {
+  if (ws->owned && ws->base) {
+    cudaError_t e = cudaFreeAsync(ws->base, st);
+    ws->base = nullptr;
+    if (e != cudaSuccess) return cuda_fail(e, "workspace: cudaFreeAsync");
+  }
+  return SSHOPM_OK;
+}
+
 int device_sms() {
   int dev = 0, sms = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) return -1;
@@ -87,11 +116,13 @@ int sshopm_create(int m, int n, sshopm_t* out) {
   if (!h) return SSHOPM_ENOMEM;
   h->L = L;
   h->launches.store(0);
+  h->hc = nullptr;
   *out = h;
   return SSHOPM_OK;
 }
 
 int sshopm_destroy(sshopm_t h) {
+  if (h) free_host_cache(h);
   delete h;
   return SSHOPM_OK;
 }
@@ -121,6 +152,12 @@ int sshopm_launch_count(sshopm_t h, int64_t* count) {
   return SSHOPM_OK;
 }
 
+int sshopm_workspace_size(sshopm_t h, int64_t N, size_t* bytes) {
+  if (!h || N < 0 || !bytes) return SSHOPM_EINVAL;
+  *bytes = workspace_bytes(h->L, N);
+  return SSHOPM_OK;
+}
+
 int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
                     float alpha, float tol, int maxit,
                     float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
@@ -131,34 +168,45 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   if (N > (1LL << 40) / S) return SSHOPM_EUNSUPPORTED;
   const Launchers* L = h->L;
   const int n = L->n;
-  const long long total = (long long)N * S;
+  cudaStream_t st = (cudaStream_t)stream;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
 
-  const int smem = (S * n * 4 <= 64 * 1024) ? S * n * 4 : 0;
-  const bool neg = alpha < 0.f;
+  const int sst = n <= 4 ? 4 : n;
+  const int smem = (S * sst * 4 <= 64 * 1024) ? S * sst * 4 : 0;
+  const int shift = alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2);
   int bps = 0;
-  cudaError_t e = L->occupancy(neg, smem, &bps);
+  cudaError_t e = L->occupancy(shift, smem, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
   if (bps < 1) bps = 1;
   if (opts && opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
-  const long long warps_full = (long long)sms * bps * 8;
-  long long ipw = (total + warps_full - 1) / warps_full;
-  if (ipw < 64) ipw = 64;                       // keep lanes busy on small problems
-  if (ipw > (1LL << 30)) return SSHOPM_EUNSUPPORTED;
-  const long long warps = (total + ipw - 1) / ipw;
-  const long long grid = (warps + 7) / 8;
+  const int chunk_tensors = (S >= 256) ? 1 : (256 + S - 1) / S;      // >= 256 items per chunk
+  const long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
+  if (n_chunks >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
+  long long grid = (long long)sms * bps;
+  if (grid * 8 > n_chunks) grid = (n_chunks + 7) / 8;
+  if (grid < 1) grid = 1;
+
+  Workspace ws;
+  int rc = acquire_workspace(L, N, opts ? opts->d_workspace : nullptr, opts ? opts->workspace_bytes : 0, st, &ws);
+  if (rc != SSHOPM_OK) return rc;
+  long long pgrid = (N + 255) / 256;
+  if (pgrid > (long long)sms * 8) pgrid = (long long)sms * 8;
+  e = L->pack(N, d_entries, ws.packed, ws.counter, (int)pgrid, st);
+  if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: pack launch"); }
 
   SolveParams p;
-  p.entries = d_entries;
+  p.packed = ws.packed;
   p.starts = d_starts;
   p.out_lambda = d_out_lambda;
   p.out_x = d_out_x;
   p.out_iters = d_out_iters;
   p.out_conv = d_out_converged;
   p.total_iters = opts ? opts->d_total_iters : nullptr;
-  p.total_items = total;
-  p.items_per_warp = ipw;
+  p.counter = ws.counter;
+  p.n_tensors = N;
+  p.n_chunks = n_chunks;
+  p.chunk_tensors = chunk_tensors;
   p.S = S;
   p.divS = make_fastdiv((uint32_t)S);
   p.alpha = alpha;
@@ -167,10 +215,10 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : L->default_refill;
   p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
   p.starts_in_smem = smem > 0 ? 1 : 0;
-  e = L->solve(p, neg, (int)grid, smem, (cudaStream_t)stream);
-  if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: launch");
-  h->launches.fetch_add(1);
-  return SSHOPM_OK;
+  e = L->solve(p, shift, (int)grid, smem, st);
+  if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
+  h->launches.fetch_add(2);
+  return release_workspace(&ws, st);
 }
 
 int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
@@ -186,14 +234,19 @@ int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x
   if (!h || N < 0) return SSHOPM_EINVAL;
   if (N == 0) return SSHOPM_OK;
   if (!d_entries || !d_x || !d_out_g || !d_out_lam) return SSHOPM_EINVAL;
+  cudaStream_t st = (cudaStream_t)stream;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_apply: no device");
   long long grid = (N + 255) / 256;
   if (grid > (long long)sms * 16) grid = (long long)sms * 16;
-  cudaError_t e = h->L->apply(N, d_entries, d_x, d_out_g, d_out_lam, (int)grid, (cudaStream_t)stream);
-  if (e != cudaSuccess) return cuda_fail(e, "sshopm_apply: launch");
-  h->launches.fetch_add(1);
-  return SSHOPM_OK;
+  Workspace ws;
+  int rc = acquire_workspace(h->L, N, nullptr, 0, st, &ws);
+  if (rc != SSHOPM_OK) return rc;
+  cudaError_t e = h->L->pack(N, d_entries, ws.packed, nullptr, (int)grid, st);
+  if (e == cudaSuccess) e = h->L->apply(N, ws.packed, d_x, d_out_g, d_out_lam, (int)grid, st);
+  if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_apply: launch"); }
+  h->launches.fetch_add(2);
+  return release_workspace(&ws, st);
 }
 
 }  // extern "C"

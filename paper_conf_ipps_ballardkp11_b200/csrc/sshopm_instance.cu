@@ -18,31 +18,41 @@ void class_index(int32_t* out) {
     for (int t = 0; t < M; ++t) out[c * M + t] = T.cls_idx[c][t];
 }
 
-cudaError_t occupancy(bool neg, int smem, int* bps) {
-  return neg ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, true>, 256, smem)
-             : cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, false>, 256, smem);
+template <int SH>
+cudaError_t occ1(int smem, int* bps) {
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH>, 256, smem);
+}
+cudaError_t occupancy(int shift, int smem, int* bps) {
+  return shift == 0 ? occ1<0>(smem, bps) : shift == 1 ? occ1<1>(smem, bps) : occ1<2>(smem, bps);
 }
 
-cudaError_t solve(const SolveParams& p, bool neg, int grid, int smem, cudaStream_t st) {
+template <int SH>
+cudaError_t solve1(const SolveParams& p, int grid, int smem, cudaStream_t st) {
   if (smem > 48 * 1024) {
-    cudaError_t e = neg ? cudaFuncSetAttribute(sshopm_solve_kernel<M, N, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)
-                        : cudaFuncSetAttribute(sshopm_solve_kernel<M, N, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(sshopm_solve_kernel<M, N, SH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
   }
-  if (neg) sshopm_solve_kernel<M, N, true><<<grid, 256, smem, st>>>(p);
-  else sshopm_solve_kernel<M, N, false><<<grid, 256, smem, st>>>(p);
+  sshopm_solve_kernel<M, N, SH><<<grid, 256, smem, st>>>(p);
+  return cudaGetLastError();
+}
+cudaError_t solve(const SolveParams& p, int shift, int grid, int smem, cudaStream_t st) {
+  return shift == 0 ? solve1<0>(p, grid, smem, st) : shift == 1 ? solve1<1>(p, grid, smem, st) : solve1<2>(p, grid, smem, st);
+}
+
+cudaError_t pack(long long n, const float* e, float4* packed, unsigned int* counter, int grid, cudaStream_t st) {
+  sshopm_pack_kernel<M, N><<<grid, 256, 0, st>>>(n, e, packed, counter);
   return cudaGetLastError();
 }
 
-cudaError_t apply(long long n_items, const float* e, const float* x, float* g, float* lam, int grid, cudaStream_t st) {
-  sshopm_apply_kernel<M, N><<<grid, 256, 0, st>>>(n_items, e, x, g, lam);
+cudaError_t apply(long long n_items, const float4* packed, const float* x, float* g, float* lam, int grid, cudaStream_t st) {
+  sshopm_apply_kernel<M, N><<<grid, 256, 0, st>>>(n_items, packed, x, g, lam);
   return cudaGetLastError();
 }
 
-const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q,
+const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
                       Sh::BFORM ? 1 : 0, 8,
-                      class_index, occupancy, solve, apply};
+                      class_index, occupancy, pack, solve, apply};
 }  // namespace
 
 #define SSHOPM_CAT2(a, b, c) get_launchers_##a##_##b

@@ -2,22 +2,23 @@
 //
 // Paper: Fig. 1 SS-HOPM, Eq. 6 / Eq. 4 kernels,
 // loop unrolling per (m, n) (Sec. V-D), data structures
-// (Sec. V-C).  Design notes: DESIGN.md "Kernels".
+// (Sec. V-C), precomputed coefficient tables shared by all
+// same-size tensors.  Design notes: DESIGN.md "Kernels".
 //
 // Mapping (differs from the paper's block-per-tensor / thread-per-start):
-//   * one lane = one (tensor, start) work item at a time; a persistent grid of
-//     warps, each owning a contiguous static range of items (tensor-major, so
-//     a warp's consecutive items share a tensor);
-//   * the whole iteration lives in registers: per-lane coefficient registers
-//     (B-form: coefficient-folded entries, or raw entries), x, lambda_prev, k;
+//   * a pack kernel rewrites each tensor's U entries once into a 16-byte
+//     aligned row of coefficient-folded words (B-form) or padded raw entries;
+//   * the solve kernel is a persistent grid of warps; one lane holds one
+//     (tensor, start) item at a time; warps claim chunks of whole tensors
+//     from a global atomic counter (dynamic load balance);
+//   * the whole iteration lives in registers: coefficients (LDG.128 from the
+//     packed row at refill), x, lambda_prev, k;
 //   * lambda = x . (A x^{M-1}) (Euler identity), so one Eq. 6 evaluation per
-//     iteration gives both kernels of Fig. 1;
+//     iteration provides both kernels of Fig. 1;
 //   * lanes that stop freeze (their state recomputes bit-identically) and the
-//     warp refills them in batches: once >= K lanes are idle it writes their
-//     results and hands them the next items of its range (warp ballot + popc,
-//     no atomics, no block barriers);
-//   * output pairs (g_0, g_1), (g_2, g_3), ... accumulate with packed FFMA2
-//     (__ffma2_rn) so the FP32 pipe is saturated at half the issue slots.
+//     warp refills them in batches once >= K lanes are idle (ballot + popc);
+//   * output pairs (g_0, g_1), ... accumulate with packed FFMA2 (__ffma2_rn),
+//     odd last output in q-pairs, so the FP32 pipe is fed at half the issue slots.
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -32,6 +33,16 @@ struct FastDiv {        // n / d for 0 <= n < 2^31, d >= 1 (Granlund-Montgomery)
 __device__ __forceinline__ uint32_t fast_div(uint32_t n, const FastDiv& f) {
   return (__umulhi(n, f.magic) + n) >> f.shift;
 }
+__device__ __forceinline__ float rsqrt_ftz(float v) {
+  float r;
+  asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(v));
+  return r;
+}
+__device__ __forceinline__ float2 f2(float a, float b) { return make_float2(a, b); }
+__device__ __forceinline__ float2 bc(float a) { return make_float2(a, a); }
+__device__ __forceinline__ float4 ldg4(const float4* p) { return __ldg(p); }
+
+constexpr int round4(int v) { return (v + 3) / 4 * 4; }
 
 template <int M, int N>
 struct Shape {
@@ -42,89 +53,128 @@ struct Shape {
   static constexpr int NP = N / 2;          // packed output pairs
   static constexpr bool ODD = (N % 2) != 0;
   static constexpr int NX = (N + 1) / 2;    // float2 slots holding x
+  static constexpr int QP = Q / 2;          // q-pairs of the odd output (leftover q handled scalar)
   // B-form keeps Q*N coefficient-folded entries per lane; raw form keeps U.
   static constexpr bool BFORM = (Q * N <= 64);
-  // register budget -> min resident blocks of 256 threads (tuned on B200)
+  static constexpr int PW_B = Q * NP * 2 + (ODD ? 2 * QP + (Q % 2) : 0);
+  static constexpr int PW = round4(BFORM ? PW_B : U);   // packed words per tensor
   static constexpr int MINB = BFORM ? (Q * N <= 32 ? 4 : 2) : (U <= 48 ? 2 : 1);
 };
 
+// ---------------------------------------------------------- pack kernel ----
+// B-form row:  [ (B_{q,2p}, B_{q,2p+1}) for q, p ] [ (B_{2t,N-1}, B_{2t+1,N-1}) for t < QP ] [B_{Q-1,N-1} if Q odd] [0 pad]
+// with B_{q,j} = ((M-1)!/q!) * a_{class(q + e_j)}   (Eq. 6 regrouped by monomial)
+// raw row:     [ a_0 .. a_{U-1} ] [0 pad]
+template <int M, int N>
+__global__ void __launch_bounds__(256)
+sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float4* __restrict__ packed,
+                   unsigned int* __restrict__ counter) {
+  using S = Shape<M, N>;
+  if (counter && blockIdx.x == 0 && threadIdx.x == 0) *counter = 0u;   // chunk counter of the following solve
+  for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n_tensors;
+       t += (long long)gridDim.x * blockDim.x) {
+    float a[S::U];
+    static_for<S::U>([&](auto c) { a[decltype(c)::value] = __ldg(entries + t * S::U + decltype(c)::value); });
+    float w[S::PW];
+#pragma unroll
+    for (int i = 0; i < S::PW; ++i) w[i] = 0.f;
+    if constexpr (S::BFORM) {
+      static_for<S::Q>([&](auto qq) {
+        constexpr int q = decltype(qq)::value;
+        constexpr float cf = (float)S::T.q_coef[q];
+        static_for<S::NP>([&](auto pp) {
+          constexpr int p = decltype(pp)::value;
+          constexpr int c0 = S::T.q_cls[q][2 * p], c1 = S::T.q_cls[q][2 * p + 1];
+          w[(q * S::NP + p) * 2 + 0] = cf * a[c0];
+          w[(q * S::NP + p) * 2 + 1] = cf * a[c1];
+        });
+        if constexpr (S::ODD) {
+          constexpr int c2 = S::T.q_cls[q][N - 1];
+          w[S::Q * S::NP * 2 + q] = cf * a[c2];
+        }
+      });
+    } else {
+#pragma unroll
+      for (int c = 0; c < S::U; ++c) w[c] = a[c];
+    }
+    float4* dst = packed + t * (S::PW / 4);
+#pragma unroll
+    for (int i = 0; i < S::PW / 4; ++i) dst[i] = make_float4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
+  }
+}
+
 // -------------------------------------------------------- coefficient regs --
 template <int M, int N, bool BF = Shape<M, N>::BFORM>
-struct Coefs;
-
-// B-form: bp[q][p] = ((M-1)!/q!) * (a_{class(q+e_{2p})}, a_{class(q+e_{2p+1})}),
-//         bs[q]    = ((M-1)!/q!) * a_{class(q+e_{N-1})} (N odd).
-template <int M, int N>
-struct Coefs<M, N, true> {
+struct Coefs {
   using S = Shape<M, N>;
-  float2 bp[S::Q][S::NP > 0 ? S::NP : 1];
-  float bs[S::Q];
+  float4 w[S::PW / 4];
 
-  __device__ __forceinline__ void load(const float* __restrict__ e) {
-    float a[S::U];
-    static_for<S::U>([&](auto c) { a[decltype(c)::value] = __ldg(e + decltype(c)::value); });
-    static_for<S::Q>([&](auto qq) {
-      constexpr int q = decltype(qq)::value;
-      constexpr float cf = (float)S::T.q_coef[q];
+  __device__ __forceinline__ void load(const float4* __restrict__ src) {
+#pragma unroll
+    for (int i = 0; i < S::PW / 4; ++i) w[i] = ldg4(src + i);
+  }
+  template <int I>
+  __device__ __forceinline__ float word() const {
+    constexpr int v = I / 4, c = I % 4;
+    if constexpr (c == 0) return w[v].x;
+    else if constexpr (c == 1) return w[v].y;
+    else if constexpr (c == 2) return w[v].z;
+    else return w[v].w;
+  }
+  template <int I>   // aligned pair of words (I even)
+  __device__ __forceinline__ float2 pair() const {
+    constexpr int v = I / 4;
+    if constexpr ((I % 4) == 0) return f2(w[v].x, w[v].y);
+    else return f2(w[v].z, w[v].w);
+  }
+
+  // g = A x^{M-1} from the Q monomials mq.
+  __device__ __forceinline__ void contract(const float (&mq)[S::Q], float2 (&gp)[S::NP > 0 ? S::NP : 1], float& gs) const {
+    if constexpr (BF) {
       static_for<S::NP>([&](auto pp) {
         constexpr int p = decltype(pp)::value;
-        constexpr int c0 = S::T.q_cls[q][2 * p], c1 = S::T.q_cls[q][2 * p + 1];
-        bp[q][p] = make_float2(cf * a[c0], cf * a[c1]);
+        gp[p] = __fmul2_rn(pair<2 * p>(), bc(mq[0]));
+      });
+      static_for<S::Q - 1>([&](auto qq) {
+        constexpr int q = decltype(qq)::value + 1;
+        static_for<S::NP>([&](auto pp) {
+          constexpr int p = decltype(pp)::value;
+          gp[p] = __ffma2_rn(pair<(q * S::NP + p) * 2>(), bc(mq[q]), gp[p]);
+        });
       });
       if constexpr (S::ODD) {
-        constexpr int c2 = S::T.q_cls[q][N - 1];
-        bs[q] = cf * a[c2];
+        constexpr int base = S::Q * S::NP * 2;
+        if constexpr (S::QP > 0) {
+          float2 h = __fmul2_rn(pair<base>(), f2(mq[0], mq[1]));
+          static_for<S::QP - 1>([&](auto tt) {
+            constexpr int t = decltype(tt)::value + 1;
+            h = __ffma2_rn(pair<base + 2 * t>(), f2(mq[2 * t], mq[2 * t + 1]), h);
+          });
+          gs = h.x + h.y;
+          if constexpr (S::Q % 2) gs = fmaf(word<base + S::Q - 1>(), mq[S::Q - 1], gs);
+        } else {
+          gs = word<base>() * mq[0];
+        }
       }
-    });
-  }
-
-  // g = A x^{M-1} from the Q monomials mq (coefficients already folded in)
-  __device__ __forceinline__ void contract(const float (&mq)[S::Q], float2 (&gp)[S::NP > 0 ? S::NP : 1], float& gs) const {
-    static_for<S::NP>([&](auto pp) {
-      constexpr int p = decltype(pp)::value;
-      gp[p] = __fmul2_rn(bp[0][p], make_float2(mq[0], mq[0]));
-    });
-    if constexpr (S::ODD) gs = bs[0] * mq[0];
-    static_for<S::Q - 1>([&](auto qq) {
-      constexpr int q = decltype(qq)::value + 1;
-      const float2 mm = make_float2(mq[q], mq[q]);
+    } else {
+      float g[N];
+      static_for<S::Q>([&](auto qq) {
+        constexpr int q = decltype(qq)::value;
+        constexpr float cf = (float)S::T.q_coef[q];
+        const float m = (cf == 1.0f) ? mq[q] : cf * mq[q];
+        static_for<N>([&](auto jj) {
+          constexpr int j = decltype(jj)::value;
+          constexpr int c = S::T.q_cls[q][j];
+          if constexpr (q == 0) g[j] = word<c>() * m;
+          else g[j] = fmaf(word<c>(), m, g[j]);
+        });
+      });
       static_for<S::NP>([&](auto pp) {
         constexpr int p = decltype(pp)::value;
-        gp[p] = __ffma2_rn(bp[q][p], mm, gp[p]);
+        gp[p] = f2(g[2 * p], g[2 * p + 1]);
       });
-      if constexpr (S::ODD) gs = fmaf(bs[q], mq[q], gs);
-    });
-  }
-};
-
-// raw form: a[c] = entry of class c; coefficients multiply the monomials.
-template <int M, int N>
-struct Coefs<M, N, false> {
-  using S = Shape<M, N>;
-  float a[S::U];
-
-  __device__ __forceinline__ void load(const float* __restrict__ e) {
-    static_for<S::U>([&](auto c) { a[decltype(c)::value] = __ldg(e + decltype(c)::value); });
-  }
-
-  __device__ __forceinline__ void contract(const float (&mq)[S::Q], float2 (&gp)[S::NP > 0 ? S::NP : 1], float& gs) const {
-    float g[N];
-    static_for<S::Q>([&](auto qq) {
-      constexpr int q = decltype(qq)::value;
-      constexpr float cf = (float)S::T.q_coef[q];
-      const float m = (cf == 1.0f) ? mq[q] : cf * mq[q];
-      static_for<N>([&](auto jj) {
-        constexpr int j = decltype(jj)::value;
-        constexpr int c = S::T.q_cls[q][j];
-        if constexpr (q == 0) g[j] = a[c] * m;
-        else g[j] = fmaf(a[c], m, g[j]);
-      });
-    });
-    static_for<S::NP>([&](auto pp) {
-      constexpr int p = decltype(pp)::value;
-      gp[p] = make_float2(g[2 * p], g[2 * p + 1]);
-    });
-    if constexpr (S::ODD) gs = g[N - 1];
+      if constexpr (S::ODD) gs = g[N - 1];
+    }
   }
 };
 
@@ -134,7 +184,7 @@ __device__ __forceinline__ float xget(const float2 (&xs)[(N + 1) / 2], int i) {
   return (i & 1) ? xs[i >> 1].y : xs[i >> 1].x;
 }
 
-// degree-(M-1) monomials x^q (Tables: lower list up to degree H, then left*right)
+// degree-(M-1) monomials x^q (lower list up to degree H, then left * right)
 template <int M, int N>
 __device__ __forceinline__ void monomials(const float2 (&xs)[(N + 1) / 2], float (&mq)[Shape<M, N>::Q]) {
   using S = Shape<M, N>;
@@ -178,21 +228,23 @@ __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&
 
 // ------------------------------------------------------------ solve kernel --
 struct SolveParams {
-  const float* entries;      // [N][U]
+  const float4* packed;      // [N][PW/4] from sshopm_pack_kernel
   const float* starts;       // [S][n] (raw; normalised in the kernel)
   float* out_lambda;         // [N][S]
   float* out_x;              // [N][S][n]
   int32_t* out_iters;        // [N][S]
   uint8_t* out_conv;         // [N][S]
   unsigned long long* total_iters;  // optional
-  long long total_items;     // N*S
-  long long items_per_warp;  // contiguous range per warp (< 2^30)
+  unsigned int* counter;     // chunk counter (zeroed by the pack kernel)
+  long long n_tensors;
+  long long n_chunks;
+  int chunk_tensors;         // tensors per chunk
   int S;
   FastDiv divS;
   float alpha, tol;
   int maxit;
   int refill_k;              // refill threshold
-  int starts_in_smem;        // 1: normalised starts cached in shared memory
+  int starts_in_smem;        // 1: normalised starts cached in shared memory (stride SSTR)
 };
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -201,11 +253,17 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return r;
 }
 
-template <int M, int N, bool NEG>
+template <int N>
+struct StartStride { static constexpr int v = (N <= 4) ? 4 : N; };
+
+// SHIFT: 0 -> alpha == 0 (xhat = g), 1 -> alpha > 0 (xhat = g + alpha x), 2 -> alpha < 0 (xhat = -(g + alpha x))
+template <int M, int N, int SHIFT>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
   using S = Shape<M, N>;
-  extern __shared__ float s_starts[];   // [S][n] normalised starts (if starts_in_smem)
+  constexpr int SST = StartStride<N>::v;
+  extern __shared__ float4 s_starts4[];
+  float* s_starts = reinterpret_cast<float*>(s_starts4);
 
   if (p.starts_in_smem) {
     for (int s = threadIdx.x; s < p.S; s += blockDim.x) {
@@ -215,90 +273,131 @@ sshopm_solve_kernel(const SolveParams p) {
       for (int j = 0; j < N; ++j) { v[j] = __ldg(p.starts + (size_t)s * N + j); nn = fmaf(v[j], v[j], nn); }
       const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
 #pragma unroll
-      for (int j = 0; j < N; ++j) s_starts[s * N + j] = v[j] * r;
+      for (int j = 0; j < SST; ++j) s_starts[s * SST + j] = (j < N) ? v[j] * r : 0.f;
     }
     __syncthreads();
   }
 
   const int lane = threadIdx.x & 31;
-  const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const long long base = gwarp * p.items_per_warp;
-  if (base >= p.total_items) return;
-  const long long span = min(p.items_per_warp, p.total_items - base);
-  const uint32_t end = (uint32_t)span;
-  const long long base_v = base / p.S;                 // tensor of the range's first item
-  const uint32_t base_s = (uint32_t)(base - base_v * p.S);
   const uint32_t ltmask = lanemask_lt();
+  const uint32_t FULL = 0xffffffffu;
+  const float alpha = (SHIFT == 2) ? -p.alpha : p.alpha;   // xhat = sgn*g + (sgn*alpha) x
+  const float tol = p.tol;
+  const int maxit = p.maxit;
+  const int S_ = p.S;
+
+  // warp-uniform chunk state
+  long long c_vox = 0;        // first tensor of the current chunk
+  uint32_t c_next = 0, c_end = 0;
+  bool exhausted = false;
 
   Coefs<M, N> cf;
   float2 xs[S::NX];
 #pragma unroll
-  for (int i = 0; i < S::NX; ++i) xs[i] = make_float2(0.f, 0.f);
+  for (int i = 0; i < S::NX; ++i) xs[i] = f2(0.f, 0.f);
   float lamp = 0.f, lam = 0.f;
   int k = 0;
   bool has = false, stop = true, conv = false;
-  uint32_t l = 0, next = 0;
+  long long item = 0;
   unsigned long long it_sum = 0;
-  const float alpha = NEG ? -p.alpha : p.alpha;   // xhat = sgn*(g + alpha x) = sgn*g + (sgn*alpha) x
 
   for (;;) {
     // ---------------- refill (warp-uniform branch) ----------------
-    const uint32_t smask = __ballot_sync(0xffffffffu, stop);
-    const int cnt = __popc(smask);
-    if ((cnt >= p.refill_k && next < end) || smask == 0xffffffffu) {
+    const uint32_t smask = __ballot_sync(FULL, stop);
+    const uint32_t cnt = __popc(smask);
+    if ((cnt >= (uint32_t)p.refill_k && !exhausted) || smask == FULL) {
       if (stop && has) {
-        const long long item = base + l;
         p.out_lambda[item] = lam;
+        float* ox = p.out_x + item * N;
 #pragma unroll
-        for (int j = 0; j < N; ++j) p.out_x[item * N + j] = xget<N>(xs, j);
+        for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
         p.out_iters[item] = k;
         p.out_conv[item] = conv ? 1 : 0;
         it_sum += (unsigned long long)k;
       }
-      const uint32_t nl = next + (uint32_t)__popc(smask & ltmask);
-      if (stop) {
-        has = nl < end;
-        if (has) {
-          l = nl;
-          const uint32_t t = base_s + l;
-          const uint32_t vq = fast_div(t, p.divS);
-          const uint32_t s = t - vq * (uint32_t)p.S;
-          cf.load(p.entries + (size_t)(base_v + vq) * S::U);
-          float v[N];
-          if (p.starts_in_smem) {
-#pragma unroll
-            for (int j = 0; j < N; ++j) v[j] = s_starts[s * N + j];
-          } else {
-            float nn = 0.f;
-#pragma unroll
-            for (int j = 0; j < N; ++j) { v[j] = __ldg(p.starts + (size_t)s * N + j); nn = fmaf(v[j], v[j], nn); }
-            const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
-#pragma unroll
-            for (int j = 0; j < N; ++j) v[j] *= r;
+      if (stop) has = false;                                 // written; refilled below if work remains
+      if (!exhausted) {
+        const uint32_t rank = __popc(smask & ltmask);
+        const uint32_t avail = c_end - c_next;             // invariant: c_next <= c_end
+        long long n_vox = 0;
+        uint32_t n_end = 0;
+        if (cnt > avail) {                                   // claim the next chunk (one atomic per warp)
+          unsigned int ch = 0;
+          if (lane == 0) ch = atomicAdd(p.counter, 1u);
+          ch = __shfl_sync(FULL, ch, 0);
+          if ((long long)ch < p.n_chunks) {
+            n_vox = (long long)ch * p.chunk_tensors;
+            const long long nt = p.n_tensors - n_vox;
+            n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
           }
+        }
+        if (stop) {
+          long long v0;
+          uint32_t t;
+          bool ok;
+          if (rank < avail) { v0 = c_vox; t = c_next + rank; ok = true; }
+          else { v0 = n_vox; t = rank - avail; ok = t < n_end; }
+          has = ok;
+          if (ok) {
+            const uint32_t vq = fast_div(t, p.divS);
+            const uint32_t s = t - vq * (uint32_t)S_;
+            item = v0 * S_ + t;
+            cf.load(p.packed + (v0 + vq) * (S::PW / 4));
+            float v[SST];
+            if (p.starts_in_smem) {
+              if constexpr (SST == 4) {
+                const float4 q4 = s_starts4[s];
+                v[0] = q4.x; v[1] = q4.y; v[2] = q4.z; v[3] = q4.w;
+              } else {
 #pragma unroll
-          for (int i = 0; i < S::NX; ++i) xs[i] = make_float2(v[2 * i], (2 * i + 1 < N) ? v[2 * i + 1] : 0.f);
-          k = 0;
-          lamp = __int_as_float(0x7fffffff);   // NaN: the first test never fires (reading R2)
+                for (int j = 0; j < SST; ++j) v[j] = s_starts[s * SST + j];
+              }
+            } else {
+              float nn = 0.f;
+#pragma unroll
+              for (int j = 0; j < N; ++j) { v[j] = __ldg(p.starts + (size_t)s * N + j); nn = fmaf(v[j], v[j], nn); }
+              const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
+#pragma unroll
+              for (int j = 0; j < N; ++j) v[j] *= r;
+            }
+#pragma unroll
+            for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], (2 * i + 1 < N) ? v[2 * i + 1] : 0.f);
+            k = 0;
+            lamp = __int_as_float(0x7fffffff);   // NaN: the first test never fires (reading R2)
+          }
+        }
+        if (cnt > avail) {
+          if (n_end == 0) exhausted = true;
+          c_vox = n_vox;
+          c_next = min(cnt - avail, n_end);                // a chunk smaller than the request is used up
+          c_end = n_end;
+        } else {
+          c_next += cnt;
         }
       }
-      next += (uint32_t)cnt;
-      if (__ballot_sync(0xffffffffu, has) == 0u) break;
+      if (__ballot_sync(FULL, has) == 0u) break;
     }
 
     // ---------------- one SS-HOPM step (Fig. 1) ----------------
     float2 gp[S::NP > 0 ? S::NP : 1];
     float gs = 0.f;
     lam = evaluate<M, N>(cf, xs, gp, gs);                       // g = A x_k^{m-1}, lam_k = x_k . g
-    conv = fabsf(lam - lamp) <= p.tol * fmaxf(1.0f, fabsf(lam)); // R2 (NaN lamp -> false)
+    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));  // R2 (NaN lamp -> false)
     // xhat = +-(g + alpha x)   (Fig. 1 lines 2-5, R5)
     float2 hp[S::NX];
     static_for<S::NP>([&](auto qq) {
       constexpr int i = decltype(qq)::value;
-      const float2 g = NEG ? make_float2(-gp[i].x, -gp[i].y) : gp[i];
-      hp[i] = __ffma2_rn(make_float2(alpha, alpha), xs[i], g);
+      if constexpr (SHIFT == 0) hp[i] = gp[i];
+      else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
+      else hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
     });
-    if constexpr (S::ODD) hp[S::NX - 1] = make_float2(fmaf(alpha, xs[S::NX - 1].x, NEG ? -gs : gs), 0.f);
+    if constexpr (S::ODD) {
+      float h;
+      if constexpr (SHIFT == 0) h = gs;
+      else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
+      else h = fmaf(alpha, xs[S::NX - 1].x, -gs);
+      hp[S::NX - 1] = f2(h, 0.f);
+    }
     float nn;
     {
       float2 t = __fmul2_rn(hp[0], hp[0]);
@@ -308,13 +407,12 @@ sshopm_solve_kernel(const SolveParams p) {
       });
       nn = t.x + t.y;
     }
-    const bool deg = !(nn > 0.f);                               // R6
-    stop = !has || conv || k >= p.maxit || deg;
+    const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
+    stop = !has || conv || k >= maxit || deg;
+    const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
     if (!stop) {
-      const float r = rsqrtf(nn);                               // line 7: x = xhat / ||xhat||
-      const float2 rr = make_float2(r, r);
 #pragma unroll
-      for (int i = 0; i < S::NX; ++i) xs[i] = __fmul2_rn(hp[i], rr);
+      for (int i = 0; i < S::NX; ++i) xs[i] = __fmul2_rn(hp[i], bc(r));
       lamp = lam;
       ++k;
     }
@@ -330,16 +428,16 @@ sshopm_solve_kernel(const SolveParams p) {
 // ------------------------------------------------------------ apply kernel --
 template <int M, int N>
 __global__ void __launch_bounds__(256)
-sshopm_apply_kernel(long long n_items, const float* __restrict__ entries, const float* __restrict__ x,
+sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const float* __restrict__ x,
                     float* __restrict__ out_g, float* __restrict__ out_lam) {
   using S = Shape<M, N>;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n_items; i += (long long)gridDim.x * blockDim.x) {
     Coefs<M, N> cf;
-    cf.load(entries + (size_t)i * S::U);
+    cf.load(packed + i * (S::PW / 4));
     float2 xs[S::NX];
 #pragma unroll
     for (int t = 0; t < S::NX; ++t)
-      xs[t] = make_float2(__ldg(x + i * N + 2 * t), (2 * t + 1 < N) ? __ldg(x + i * N + 2 * t + 1) : 0.f);
+      xs[t] = f2(__ldg(x + i * N + 2 * t), (2 * t + 1 < N) ? __ldg(x + i * N + 2 * t + 1) : 0.f);
     float2 gp[S::NP > 0 ? S::NP : 1];
     float gs = 0.f;
     const float lam = evaluate<M, N>(cf, xs, gp, gs);

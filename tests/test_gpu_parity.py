@@ -219,6 +219,16 @@ def test_run_host_matches_device_path(dev):
     assert out["total_iters"] == int(it.cpu().numpy().sum())
 
 
+@pytest.mark.parametrize("V,S", [(1, 1), (3, 1), (5, 7), (40, 2), (2, 300)])
+def test_tiny_chunks(dev, V, S):
+    """Chunks smaller than a warp's request (S * tensors < 32) must not overrun (regression)."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 77, V, 0)
+    st = syn.gen_starts(S, n, 1)
+    gpu = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
+    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, gpu), max_sensitive=0.02)
+
+
 def test_empty_and_tiny(dev):
     m, n = 4, 3
     s = sh.Solver(m, n)
