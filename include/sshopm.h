@@ -98,11 +98,12 @@ int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const flo
                  float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
                  void* stream);
 
-/* Device workspace needed by sshopm_solve_ex for N tensors (bytes): a 256-byte
- * header (work counter) plus one 16-byte aligned packed coefficient row per
- * tensor (precomputed coefficients).  sshopm_solve
- * and sshopm_apply allocate it themselves (cudaMallocAsync on the stream). */
-int sshopm_workspace_size(sshopm_t h, int64_t N, size_t* bytes);
+/* Device workspace needed by sshopm_solve_ex for N tensors and S starts
+ * (bytes): a 256-byte header (work counter), the S normalised starts and one
+ * 16-byte aligned packed coefficient row per tensor (precomputed
+ * coefficients).  sshopm_solve and sshopm_apply allocate it
+ * themselves (cudaMallocAsync / cudaFreeAsync on the stream). */
+int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes);
 
 /* Tuning / instrumentation knobs for sshopm_solve_ex (0 / NULL = library default). */
 typedef struct {

@@ -59,7 +59,7 @@ def lib():
         "sshopm_apply": (I, [P, I64, P, P, P, P, P]),
         "sshopm_run_host": (I, [P, I64, P, I, P, F, F, I, F, F, I, P, P, P, P, P, P, P, P, P, I64, P]),
         "sshopm_launch_count": (I, [P, ctypes.POINTER(I64)]),
-        "sshopm_workspace_size": (I, [P, I64, ctypes.POINTER(ctypes.c_size_t)]),
+        "sshopm_workspace_size": (I, [P, I64, I, ctypes.POINTER(ctypes.c_size_t)]),
         "sshopm_status_string": (ctypes.c_char_p, [I]),
         "sshopm_last_cuda_error": (ctypes.c_char_p, []),
         "sshopm_supported_shapes": (ctypes.c_char_p, []),
@@ -144,13 +144,13 @@ class Solver:
         _check(lib().sshopm_class_index(self._h, out.ctypes.data_as(ctypes.c_void_p)), "sshopm_class_index")
         return out
 
-    def workspace_size(self, N):
+    def workspace_size(self, N, S):
         b = ctypes.c_size_t()
-        _check(lib().sshopm_workspace_size(self._h, int(N), ctypes.byref(b)), "sshopm_workspace_size")
+        _check(lib().sshopm_workspace_size(self._h, int(N), int(S), ctypes.byref(b)), "sshopm_workspace_size")
         return b.value
 
-    def _workspace(self, N, device):
-        need = self.workspace_size(N)
+    def _workspace(self, N, S, device):
+        need = self.workspace_size(N, S)
         ws = self._ws
         if ws is None or ws.device != device or ws.numel() < need:
             torch = _torch()
@@ -180,7 +180,7 @@ class Solver:
         lam, x, it, cv = out
         args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
                 _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
-        wsp, wsb = self._workspace(N, dev) if N > 0 else (None, 0)
+        wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
         opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb)
         if total_iters is not None:
             if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:

@@ -27,7 +27,7 @@ LIB = os.path.join(LIBDIR, "libsshopm.so")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
-              "-I" + INCLUDE, "-I" + CSRC] + ARCH
+              "-I" + INCLUDE, "-I" + CSRC] + ARCH + os.environ.get("SSHOPM_NVCC_EXTRA", "").split()
 
 
 def nvcc():

@@ -21,11 +21,12 @@ int device_sms();
 struct Workspace {
   void* base = nullptr;
   unsigned int* counter = nullptr;   // 256-byte header: chunk counter of the solve kernel
+  float* starts_n = nullptr;         // [S][round4(n)] normalised starts (256-byte aligned region)
   float4* packed = nullptr;          // [N][PW/4] packed coefficient rows
   bool owned = false;
 };
-size_t workspace_bytes(const Launchers* L, int64_t N);
-int acquire_workspace(const Launchers* L, int64_t N, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws);
+size_t workspace_bytes(const Launchers* L, int64_t N, int S);
+int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws);
 int release_workspace(Workspace* ws, cudaStream_t st);
 int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
                float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,

@@ -118,7 +118,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
       CK(cudaMalloc(&s.ox, sizeof(float) * chunk * kmax * n), "run_host: malloc");
       CK(cudaMalloc(&s.mult, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
       CK(cudaMalloc(&s.rep, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
-      s.ws_bytes = workspace_bytes(h->L, chunk);
+      s.ws_bytes = workspace_bytes(h->L, chunk, S);
       CK(cudaMalloc(&s.ws, s.ws_bytes), "run_host: malloc");
     }
     c->chunk = chunk;

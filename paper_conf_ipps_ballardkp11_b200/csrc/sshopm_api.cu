@@ -44,10 +44,17 @@ FastDiv make_fastdiv(uint32_t d) {
   return f;
 }
 
-size_t workspace_bytes(const Launchers* L, int64_t N) { return 256 + (size_t)N * (size_t)L->PW * 4; }
+static size_t starts_region(const Launchers* L, int S) {
+  const size_t b = (size_t)S * (size_t)((L->n + 3) / 4 * 4) * 4;
+  return (b + 255) / 256 * 256;
+}
 
-int acquire_workspace(const Launchers* L, int64_t N, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws) {
-  const size_t need = workspace_bytes(L, N);
+size_t workspace_bytes(const Launchers* L, int64_t N, int S) {
+  return 256 + starts_region(L, S) + (size_t)N * (size_t)L->PW * 4;
+}
+
+int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws) {
+  const size_t need = workspace_bytes(L, N, S);
   ws->owned = false;
   void* base = user;
   if (!user || user_bytes < need || ((uintptr_t)user & 255)) {
@@ -60,7 +67,8 @@ int acquire_workspace(const Launchers* L, int64_t N, void* user, size_t user_byt
   }
   ws->base = base;
   ws->counter = reinterpret_cast<unsigned int*>(base);
-  ws->packed = reinterpret_cast<float4*>(reinterpret_cast<char*>(base) + 256);
+  ws->starts_n = reinterpret_cast<float*>(reinterpret_cast<char*>(base) + 256);
+  ws->packed = reinterpret_cast<float4*>(reinterpret_cast<char*>(base) + 256 + starts_region(L, S));
   return SSHOPM_OK;
 }
 
@@ -152,9 +160,9 @@ int sshopm_launch_count(sshopm_t h, int64_t* count) {
   return SSHOPM_OK;
 }
 
-int sshopm_workspace_size(sshopm_t h, int64_t N, size_t* bytes) {
-  if (!h || N < 0 || !bytes) return SSHOPM_EINVAL;
-  *bytes = workspace_bytes(h->L, N);
+int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes) {
+  if (!h || N < 0 || S < 0 || !bytes) return SSHOPM_EINVAL;
+  *bytes = workspace_bytes(h->L, N, S);
   return SSHOPM_OK;
 }
 
@@ -167,16 +175,14 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   if (!d_entries || !d_starts || !d_out_lambda || !d_out_x || !d_out_iters || !d_out_converged) return SSHOPM_EINVAL;
   if (N > (1LL << 40) / S) return SSHOPM_EUNSUPPORTED;
   const Launchers* L = h->L;
-  const int n = L->n;
   cudaStream_t st = (cudaStream_t)stream;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
 
-  const int sst = n <= 4 ? 4 : n;
-  const int smem = (S * sst * 4 <= 64 * 1024) ? S * sst * 4 : 0;
   const int shift = alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2);
+  const bool wide = (long long)N * S >= (1LL << 31) - (1LL << 20);
   int bps = 0;
-  cudaError_t e = L->occupancy(shift, smem, &bps);
+  cudaError_t e = L->occupancy(shift, wide, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
   if (bps < 1) bps = 1;
   if (opts && opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
@@ -188,16 +194,16 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   if (grid < 1) grid = 1;
 
   Workspace ws;
-  int rc = acquire_workspace(L, N, opts ? opts->d_workspace : nullptr, opts ? opts->workspace_bytes : 0, st, &ws);
+  int rc = acquire_workspace(L, N, S, opts ? opts->d_workspace : nullptr, opts ? opts->workspace_bytes : 0, st, &ws);
   if (rc != SSHOPM_OK) return rc;
-  long long pgrid = (N + 255) / 256;
+  long long pgrid = ((N > S ? N : S) + 255) / 256;
   if (pgrid > (long long)sms * 8) pgrid = (long long)sms * 8;
-  e = L->pack(N, d_entries, ws.packed, ws.counter, (int)pgrid, st);
+  e = L->pack(N, d_entries, ws.packed, ws.counter, S, d_starts, ws.starts_n, (int)pgrid, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: pack launch"); }
 
   SolveParams p;
   p.packed = ws.packed;
-  p.starts = d_starts;
+  p.starts_n = reinterpret_cast<const float4*>(ws.starts_n);
   p.out_lambda = d_out_lambda;
   p.out_x = d_out_x;
   p.out_iters = d_out_iters;
@@ -214,8 +220,7 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   p.maxit = maxit;
   int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : L->default_refill;
   p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
-  p.starts_in_smem = smem > 0 ? 1 : 0;
-  e = L->solve(p, shift, (int)grid, smem, st);
+  e = L->solve(p, shift, wide, (int)grid, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
   h->launches.fetch_add(2);
   return release_workspace(&ws, st);
@@ -240,9 +245,9 @@ int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x
   long long grid = (N + 255) / 256;
   if (grid > (long long)sms * 16) grid = (long long)sms * 16;
   Workspace ws;
-  int rc = acquire_workspace(h->L, N, nullptr, 0, st, &ws);
+  int rc = acquire_workspace(h->L, N, 0, nullptr, 0, st, &ws);
   if (rc != SSHOPM_OK) return rc;
-  cudaError_t e = h->L->pack(N, d_entries, ws.packed, nullptr, (int)grid, st);
+  cudaError_t e = h->L->pack(N, d_entries, ws.packed, nullptr, 0, nullptr, nullptr, (int)grid, st);
   if (e == cudaSuccess) e = h->L->apply(N, ws.packed, d_x, d_out_g, d_out_lam, (int)grid, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_apply: launch"); }
   h->launches.fetch_add(2);

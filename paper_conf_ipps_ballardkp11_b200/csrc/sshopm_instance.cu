@@ -18,29 +18,28 @@ void class_index(int32_t* out) {
     for (int t = 0; t < M; ++t) out[c * M + t] = T.cls_idx[c][t];
 }
 
-template <int SH>
-cudaError_t occ1(int smem, int* bps) {
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH>, 256, smem);
+template <int SH, bool W>
+cudaError_t occ1(int* bps) {
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W>, 256, 0);
 }
-cudaError_t occupancy(int shift, int smem, int* bps) {
-  return shift == 0 ? occ1<0>(smem, bps) : shift == 1 ? occ1<1>(smem, bps) : occ1<2>(smem, bps);
+cudaError_t occupancy(int shift, bool wide, int* bps) {
+  if (wide) return shift == 0 ? occ1<0, true>(bps) : shift == 1 ? occ1<1, true>(bps) : occ1<2, true>(bps);
+  return shift == 0 ? occ1<0, false>(bps) : shift == 1 ? occ1<1, false>(bps) : occ1<2, false>(bps);
 }
 
-template <int SH>
-cudaError_t solve1(const SolveParams& p, int grid, int smem, cudaStream_t st) {
-  if (smem > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(sshopm_solve_kernel<M, N, SH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-  }
-  sshopm_solve_kernel<M, N, SH><<<grid, 256, smem, st>>>(p);
+template <int SH, bool W>
+cudaError_t solve1(const SolveParams& p, int grid, cudaStream_t st) {
+  sshopm_solve_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
   return cudaGetLastError();
 }
-cudaError_t solve(const SolveParams& p, int shift, int grid, int smem, cudaStream_t st) {
-  return shift == 0 ? solve1<0>(p, grid, smem, st) : shift == 1 ? solve1<1>(p, grid, smem, st) : solve1<2>(p, grid, smem, st);
+cudaError_t solve(const SolveParams& p, int shift, bool wide, int grid, cudaStream_t st) {
+  if (wide) return shift == 0 ? solve1<0, true>(p, grid, st) : shift == 1 ? solve1<1, true>(p, grid, st) : solve1<2, true>(p, grid, st);
+  return shift == 0 ? solve1<0, false>(p, grid, st) : shift == 1 ? solve1<1, false>(p, grid, st) : solve1<2, false>(p, grid, st);
 }
 
-cudaError_t pack(long long n, const float* e, float4* packed, unsigned int* counter, int grid, cudaStream_t st) {
-  sshopm_pack_kernel<M, N><<<grid, 256, 0, st>>>(n, e, packed, counter);
+cudaError_t pack(long long n, const float* e, float4* packed, unsigned int* counter, int n_starts, const float* starts,
+                 float* starts_n, int grid, cudaStream_t st) {
+  sshopm_pack_kernel<M, N><<<grid, 256, 0, st>>>(n, e, packed, counter, n_starts, starts, starts_n);
   return cudaGetLastError();
 }
 
@@ -51,7 +50,7 @@ cudaError_t apply(long long n_items, const float4* packed, const float* x, float
 
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
-                      Sh::BFORM ? 1 : 0, 8,
+                      Sh::BFORM ? 1 : 0, 10,
                       class_index, occupancy, pack, solve, apply};
 }  // namespace
 

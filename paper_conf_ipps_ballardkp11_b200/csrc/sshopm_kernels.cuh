@@ -22,6 +22,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <type_traits>
 #include "symm_tables.cuh"
 
 namespace sshopm {
@@ -43,6 +44,9 @@ __device__ __forceinline__ float2 bc(float a) { return make_float2(a, a); }
 __device__ __forceinline__ float4 ldg4(const float4* p) { return __ldg(p); }
 
 constexpr int round4(int v) { return (v + 3) / 4 * 4; }
+#ifndef SSHOPM_STEPS
+#define SSHOPM_STEPS 2
+#endif
 
 template <int M, int N>
 struct Shape {
@@ -68,9 +72,21 @@ struct Shape {
 template <int M, int N>
 __global__ void __launch_bounds__(256)
 sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float4* __restrict__ packed,
-                   unsigned int* __restrict__ counter) {
+                   unsigned int* __restrict__ counter, int n_starts, const float* __restrict__ starts,
+                   float* __restrict__ starts_n) {
   using S = Shape<M, N>;
   if (counter && blockIdx.x == 0 && threadIdx.x == 0) *counter = 0u;   // chunk counter of the following solve
+  // normalised starts x_0 = s / ||s|| in FP32 (reading R7), rows padded to SST floats
+  constexpr int SST = round4(N);
+  for (int s = blockIdx.x * blockDim.x + threadIdx.x; s < n_starts; s += gridDim.x * blockDim.x) {
+    float v[N];
+    float nn = 0.f;
+#pragma unroll
+    for (int j = 0; j < N; ++j) { v[j] = starts[(size_t)s * N + j]; nn = fmaf(v[j], v[j], nn); }
+    const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
+#pragma unroll
+    for (int j = 0; j < SST; ++j) starts_n[(size_t)s * SST + j] = (j < N) ? v[j] * r : 0.f;
+  }
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n_tensors;
        t += (long long)gridDim.x * blockDim.x) {
     float a[S::U];
@@ -203,6 +219,28 @@ __device__ __forceinline__ void monomials(const float2 (&xs)[(N + 1) / 2], float
   });
 }
 
+// (4,3): the paper's hand-unrolled case (Sec. V-D), paired for FFMA2/FMUL2.
+// x is held as (x0, x1), (x2, x1) so every degree-2 and degree-3 monomial pair
+// is one FMUL2 (8 instead of 16 FMUL); order = lex order of Tables<4,3>.
+template <int M, int N>
+struct X21 { static constexpr bool v = (M == 4 && N == 3); };
+
+template <>
+__device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
+  const float2 x01 = xs[0], x21 = xs[1];
+  const float2 x12 = f2(x21.y, x21.x);
+  const float2 s0 = __fmul2_rn(bc(x01.x), x01);   // (x0x0, x0x1)
+  const float2 s1 = __fmul2_rn(x01, x21);         // (x0x2, x1x1)
+  const float2 s2 = __fmul2_rn(bc(x21.x), x12);   // (x2x1, x2x2)
+  const float2 m01 = __fmul2_rn(bc(x01.x), s0);   // 000 001
+  const float2 m23 = __fmul2_rn(bc(x01.x), s1);   // 002 011
+  const float2 m45 = __fmul2_rn(bc(x01.x), s2);   // 012 022
+  const float2 m67 = __fmul2_rn(bc(s1.y), x12);   // 111 112
+  const float2 m89 = __fmul2_rn(bc(s2.y), x12);   // 122 222
+  mq[0] = m01.x; mq[1] = m01.y; mq[2] = m23.x; mq[3] = m23.y; mq[4] = m45.x;
+  mq[5] = m45.y; mq[6] = m67.x; mq[7] = m67.y; mq[8] = m89.x; mq[9] = m89.y;
+}
+
 // g = A x^{M-1} (pairs gp, odd tail gs) and lambda = x . g
 template <int M, int N>
 __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&xs)[(N + 1) / 2],
@@ -229,7 +267,7 @@ __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&
 // ------------------------------------------------------------ solve kernel --
 struct SolveParams {
   const float4* packed;      // [N][PW/4] from sshopm_pack_kernel
-  const float* starts;       // [S][n] (raw; normalised in the kernel)
+  const float4* starts_n;    // [S][SST/4] normalised starts from sshopm_pack_kernel
   float* out_lambda;         // [N][S]
   float* out_x;              // [N][S][n]
   int32_t* out_iters;        // [N][S]
@@ -244,7 +282,6 @@ struct SolveParams {
   float alpha, tol;
   int maxit;
   int refill_k;              // refill threshold
-  int starts_in_smem;        // 1: normalised starts cached in shared memory (stride SSTR)
 };
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -253,30 +290,16 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return r;
 }
 
-template <int N>
-struct StartStride { static constexpr int v = (N <= 4) ? 4 : N; };
-
 // SHIFT: 0 -> alpha == 0 (xhat = g), 1 -> alpha > 0 (xhat = g + alpha x), 2 -> alpha < 0 (xhat = -(g + alpha x))
-template <int M, int N, int SHIFT>
+// WIDE: 64-bit item indices (N*S >= 2^31); otherwise 32-bit index arithmetic.
+template <int M, int N, int SHIFT, bool WIDE>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
+  constexpr int STEPS = SSHOPM_STEPS;        // SS-HOPM steps between refill checks
   using S = Shape<M, N>;
-  constexpr int SST = StartStride<N>::v;
-  extern __shared__ float4 s_starts4[];
-  float* s_starts = reinterpret_cast<float*>(s_starts4);
-
-  if (p.starts_in_smem) {
-    for (int s = threadIdx.x; s < p.S; s += blockDim.x) {
-      float v[N];
-      float nn = 0.f;
-#pragma unroll
-      for (int j = 0; j < N; ++j) { v[j] = __ldg(p.starts + (size_t)s * N + j); nn = fmaf(v[j], v[j], nn); }
-      const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
-#pragma unroll
-      for (int j = 0; j < SST; ++j) s_starts[s * SST + j] = (j < N) ? v[j] * r : 0.f;
-    }
-    __syncthreads();
-  }
+  using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
+  constexpr int SST4 = round4(N) / 4;
+  constexpr bool XL = X21<M, N>::v;
 
   const int lane = threadIdx.x & 31;
   const uint32_t ltmask = lanemask_lt();
@@ -284,10 +307,10 @@ sshopm_solve_kernel(const SolveParams p) {
   const float alpha = (SHIFT == 2) ? -p.alpha : p.alpha;   // xhat = sgn*g + (sgn*alpha) x
   const float tol = p.tol;
   const int maxit = p.maxit;
-  const int S_ = p.S;
+  const uint32_t S_ = (uint32_t)p.S;
 
   // warp-uniform chunk state
-  long long c_vox = 0;        // first tensor of the current chunk
+  Idx c_vox = 0;              // first tensor of the current chunk
   uint32_t c_next = 0, c_end = 0;
   bool exhausted = false;
 
@@ -298,7 +321,7 @@ sshopm_solve_kernel(const SolveParams p) {
   float lamp = 0.f, lam = 0.f;
   int k = 0;
   bool has = false, stop = true, conv = false;
-  long long item = 0;
+  Idx item = 0;
   unsigned long long it_sum = 0;
 
   for (;;) {
@@ -306,66 +329,55 @@ sshopm_solve_kernel(const SolveParams p) {
     const uint32_t smask = __ballot_sync(FULL, stop);
     const uint32_t cnt = __popc(smask);
     if ((cnt >= (uint32_t)p.refill_k && !exhausted) || smask == FULL) {
-      if (stop && has) {
-        p.out_lambda[item] = lam;
-        float* ox = p.out_x + item * N;
-#pragma unroll
-        for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
-        p.out_iters[item] = k;
-        p.out_conv[item] = conv ? 1 : 0;
-        it_sum += (unsigned long long)k;
-      }
-      if (stop) has = false;                                 // written; refilled below if work remains
+      uint32_t avail = 0, n_end = 0;
+      Idx n_vox = 0;
       if (!exhausted) {
-        const uint32_t rank = __popc(smask & ltmask);
-        const uint32_t avail = c_end - c_next;             // invariant: c_next <= c_end
-        long long n_vox = 0;
-        uint32_t n_end = 0;
-        if (cnt > avail) {                                   // claim the next chunk (one atomic per warp)
+        avail = c_end - c_next;                            // invariant: c_next <= c_end
+        if (cnt > avail) {                                 // claim the next chunk (one atomic per warp)
           unsigned int ch = 0;
           if (lane == 0) ch = atomicAdd(p.counter, 1u);
           ch = __shfl_sync(FULL, ch, 0);
           if ((long long)ch < p.n_chunks) {
-            n_vox = (long long)ch * p.chunk_tensors;
-            const long long nt = p.n_tensors - n_vox;
+            n_vox = (Idx)ch * (Idx)p.chunk_tensors;
+            const long long nt = p.n_tensors - (long long)n_vox;
             n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
           }
         }
-        if (stop) {
-          long long v0;
-          uint32_t t;
-          bool ok;
-          if (rank < avail) { v0 = c_vox; t = c_next + rank; ok = true; }
-          else { v0 = n_vox; t = rank - avail; ok = t < n_end; }
-          has = ok;
-          if (ok) {
-            const uint32_t vq = fast_div(t, p.divS);
-            const uint32_t s = t - vq * (uint32_t)S_;
-            item = v0 * S_ + t;
-            cf.load(p.packed + (v0 + vq) * (S::PW / 4));
-            float v[SST];
-            if (p.starts_in_smem) {
-              if constexpr (SST == 4) {
-                const float4 q4 = s_starts4[s];
-                v[0] = q4.x; v[1] = q4.y; v[2] = q4.z; v[3] = q4.w;
-              } else {
+      }
+      if (stop) {
+        if (has) {
+          p.out_lambda[item] = lam;
+          float* ox = p.out_x + (size_t)item * N;            // one 64-bit row address, immediate offsets
 #pragma unroll
-                for (int j = 0; j < SST; ++j) v[j] = s_starts[s * SST + j];
-              }
-            } else {
-              float nn = 0.f;
-#pragma unroll
-              for (int j = 0; j < N; ++j) { v[j] = __ldg(p.starts + (size_t)s * N + j); nn = fmaf(v[j], v[j], nn); }
-              const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
-#pragma unroll
-              for (int j = 0; j < N; ++j) v[j] *= r;
-            }
-#pragma unroll
-            for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], (2 * i + 1 < N) ? v[2 * i + 1] : 0.f);
-            k = 0;
-            lamp = __int_as_float(0x7fffffff);   // NaN: the first test never fires (reading R2)
-          }
+          for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
+          p.out_iters[item] = k;
+          p.out_conv[item] = conv ? 1 : 0;
+          it_sum += (unsigned long long)k;
         }
+        const uint32_t rank = __popc(smask & ltmask);
+        const bool cur = rank < avail;
+        const Idx v0 = cur ? c_vox : n_vox;
+        const uint32_t t = cur ? c_next + rank : rank - avail;
+        has = !exhausted && (cur || t < n_end);
+        if (has) {
+          const uint32_t vq = fast_div(t, p.divS);
+          const uint32_t s = t - vq * S_;
+          item = v0 * (Idx)S_ + (Idx)t;
+          cf.load(p.packed + (v0 + (Idx)vq) * (Idx)(S::PW / 4));
+          float v[4 * SST4];
+#pragma unroll
+          for (int i = 0; i < SST4; ++i) {
+            const float4 q4 = ldg4(p.starts_n + s * SST4 + i);
+            v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
+          }
+#pragma unroll
+          for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
+          if constexpr (XL) xs[1].y = v[1];                // (x2, x1) layout
+          k = 0;
+          lamp = __int_as_float(0x7fffffff);               // NaN: the first test never fires (reading R2)
+        }
+      }
+      if (!exhausted) {
         if (cnt > avail) {
           if (n_end == 0) exhausted = true;
           c_vox = n_vox;
@@ -378,43 +390,59 @@ sshopm_solve_kernel(const SolveParams p) {
       if (__ballot_sync(FULL, has) == 0u) break;
     }
 
-    // ---------------- one SS-HOPM step (Fig. 1) ----------------
-    float2 gp[S::NP > 0 ? S::NP : 1];
-    float gs = 0.f;
-    lam = evaluate<M, N>(cf, xs, gp, gs);                       // g = A x_k^{m-1}, lam_k = x_k . g
-    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));  // R2 (NaN lamp -> false)
-    // xhat = +-(g + alpha x)   (Fig. 1 lines 2-5, R5)
-    float2 hp[S::NX];
-    static_for<S::NP>([&](auto qq) {
-      constexpr int i = decltype(qq)::value;
-      if constexpr (SHIFT == 0) hp[i] = gp[i];
-      else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
-      else hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
-    });
-    if constexpr (S::ODD) {
-      float h;
-      if constexpr (SHIFT == 0) h = gs;
-      else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
-      else h = fmaf(alpha, xs[S::NX - 1].x, -gs);
-      hp[S::NX - 1] = f2(h, 0.f);
-    }
-    float nn;
-    {
-      float2 t = __fmul2_rn(hp[0], hp[0]);
-      static_for<S::NX - 1>([&](auto qq) {
-        constexpr int i = decltype(qq)::value + 1;
-        t = __ffma2_rn(hp[i], hp[i], t);
-      });
-      nn = t.x + t.y;
-    }
-    const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
-    stop = !has || conv || k >= maxit || deg;
-    const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
-    if (!stop) {
+    // ---------------- SS-HOPM steps (Fig. 1), STEPS per refill check ----------------
 #pragma unroll
-      for (int i = 0; i < S::NX; ++i) xs[i] = __fmul2_rn(hp[i], bc(r));
-      lamp = lam;
-      ++k;
+    for (int rep = 0; rep < STEPS; ++rep) {
+      float2 gp[S::NP > 0 ? S::NP : 1];
+      float gs = 0.f;
+      lam = evaluate<M, N>(cf, xs, gp, gs);                       // g = A x_k^{m-1}, lam_k = x_k . g
+      conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));  // R2 (NaN lamp -> false)
+      // xhat = +-(g + alpha x)   (Fig. 1 lines 2-5, R5)
+      float2 hp[S::NX];
+      static_for<S::NP>([&](auto qq) {
+        constexpr int i = decltype(qq)::value;
+        if constexpr (SHIFT == 0) hp[i] = gp[i];
+        else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
+        else hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
+      });
+      if constexpr (S::ODD) {
+        float h;
+        if constexpr (SHIFT == 0) h = gs;
+        else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
+        else h = fmaf(alpha, xs[S::NX - 1].x, -gs);
+        hp[S::NX - 1] = f2(h, 0.f);
+      }
+      float nn;
+      {
+        float2 t = __fmul2_rn(hp[0], hp[0]);
+        static_for<S::NX - 1>([&](auto qq) {
+          constexpr int i = decltype(qq)::value + 1;
+          if constexpr (S::ODD && i == S::NX - 1) t.x = fmaf(hp[i].x, hp[i].x, t.x);
+          else t = __ffma2_rn(hp[i], hp[i], t);
+        });
+        nn = t.x + t.y;
+      }
+      const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
+      stop = !has || conv || k >= maxit || deg;
+      const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
+      // freeze stopped lanes by selection (no branch): x, lambda_prev, k keep their values
+      if constexpr (XL) {
+        const float2 n01 = __fmul2_rn(hp[0], bc(r));
+        const float n2 = hp[1].x * r;
+        xs[0].x = stop ? xs[0].x : n01.x;
+        xs[0].y = stop ? xs[0].y : n01.y;
+        xs[1].x = stop ? xs[1].x : n2;
+        xs[1].y = xs[0].y;
+      } else {
+#pragma unroll
+        for (int i = 0; i < S::NX; ++i) {
+          const float2 nx = __fmul2_rn(hp[i], bc(r));
+          xs[i].x = stop ? xs[i].x : nx.x;
+          xs[i].y = stop ? xs[i].y : nx.y;
+        }
+      }
+      lamp = stop ? lamp : lam;
+      k += stop ? 0 : 1;
     }
   }
 
@@ -438,6 +466,7 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
 #pragma unroll
     for (int t = 0; t < S::NX; ++t)
       xs[t] = f2(__ldg(x + i * N + 2 * t), (2 * t + 1 < N) ? __ldg(x + i * N + 2 * t + 1) : 0.f);
+    if constexpr (X21<M, N>::v) xs[1].y = xs[0].y;
     float2 gp[S::NP > 0 ? S::NP : 1];
     float gs = 0.f;
     const float lam = evaluate<M, N>(cf, xs, gp, gs);
