@@ -186,6 +186,7 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_ballardkp11_b200 as sh
+    from paper_conf_ipps_ballardkp11_b200 import sharding as SH
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -196,7 +197,9 @@ def main():
     U = solver.U
 
     # inputs: this rank's tensor range (counter-based generator -> shard invariant), resident in HBM
-    ent_h = syn.gen_voxels(m, n, rank * Nloc, Nloc, seed=0)
+    first, count = SH.shard_range(Nloc * world, rank, world)
+    assert count == Nloc
+    ent_h = syn.gen_voxels(m, n, first, Nloc, seed=0)
     st_h = syn.gen_starts(S, n, seed=0)
     ent = torch.from_numpy(ent_h).to(dev)
     st = torch.from_numpy(st_h).to(dev)
@@ -204,17 +207,9 @@ def main():
     xo = torch.empty((Nloc, S, n), dtype=torch.float32, device=dev)
     it = torch.empty((Nloc, S), dtype=torch.int32, device=dev)
     cv = torch.empty((Nloc, S), dtype=torch.uint8, device=dev)
-    # dedup records packed in one buffer so a single collective moves them
-    rec_words = Nloc * (1 + KMAX * (n + 3))
-    rec = torch.empty(rec_words, dtype=torch.int32, device=dev)
-    o = 0
-    views = []
-    for shape, dt in [((Nloc,), torch.int32), ((Nloc, KMAX), torch.float32), ((Nloc, KMAX, n), torch.float32),
-                      ((Nloc, KMAX), torch.int32), ((Nloc, KMAX), torch.int32)]:
-        cnt = int(np.prod(shape))
-        views.append(rec[o:o + cnt].view(dt).view(shape))
-        o += cnt
-    gathered = [torch.empty_like(rec) for _ in range(world)] if (world > 1 and rank == 0) else None
+    # dedup records packed in one int32 buffer so a single collective moves them (sharding.py)
+    rec = torch.empty(SH.record_words(Nloc, KMAX, n), dtype=torch.int32, device=dev)
+    views = SH.record_views(rec, Nloc, KMAX, n)
     titers = torch.zeros(1, dtype=torch.int64, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
@@ -226,7 +221,7 @@ def main():
                      refill_threshold=a.refill, total_iters=titers if count_iters else None)
         solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
         if world > 1:
-            dist.gather(rec, gathered, dst=0)
+            SH.gather_records(rec, rank, world)
 
     for _ in range(max(a.warmup, 3)):
         step()
@@ -250,7 +245,7 @@ def main():
             e1.record(stream)
             solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
             if world > 1:
-                dist.gather(rec, gathered, dst=0)
+                SH.gather_records(rec, rank, world)
             e2.record(stream)
         torch.cuda.synchronize()
     if world > 1:
@@ -307,7 +302,7 @@ def main():
         return
 
     F = solver.paper_flops_per_iter
-    Fx = solver.exec_flops_per_iter
+    Fx = solver.exec_flops_per_iter - (2 * n if cfg["alpha"] == 0 else 0)   # alpha = 0: no shift flops
     T = tot_ms / 1e3
     value = F * iters_all * a.steps / T / 1e9
     vps = Nloc * world * a.steps / T
@@ -347,7 +342,8 @@ def main():
                      "frac": achieved / peak_tflops, "traffic": traffic,
                      "kernel": f"sshopm_solve_kernel<{m},{n}>",
                      "peak_basis": f"{sms} SM x 128 FP32 lanes x 2 x {fmax:.0f} MHz (sm_max_mhz)",
-                     "flops_per_update": Fx},
+                     "flops_per_update": Fx,
+                     "flops_note": "algorithmic FP32 flops per (tensor,start,update): monomials + 2*T1 + lambda + shift + norm + scale (DESIGN.md 7)"},
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,
