@@ -267,6 +267,16 @@ static cudaError_t launch_dedup(const DedupParams& p, int grid, int block, int s
   return cudaGetLastError();
 }
 
+template <int NN, bool EVEN>
+static cudaError_t launch_dedup128(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup128_kernel<NN, EVEN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+  }
+  sshopm_dedup128_kernel<NN, EVEN><<<grid, block, smem, st>>>(p);
+  return cudaGetLastError();
+}
+
 int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
                float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
                int32_t* d_rep, cudaStream_t st) {
@@ -277,7 +287,9 @@ int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, cons
   const int n = L->n;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_dedup: no device");
-  const int per_warp = dedup_smem_words(S, n) * 4;
+  const bool fast = (S == 128) && n <= 8 &&
+                    ((uintptr_t)d_lambda % 16 == 0) && ((uintptr_t)d_x % 16 == 0) && ((uintptr_t)d_conv % 4 == 0);
+  const int per_warp = fast ? 128 * (n + 3) * 4 : dedup_smem_words(S, n) * 4;
   int wpb = (96 * 1024) / per_warp;
   if (wpb > 8) wpb = 8;
   if (wpb < 1) wpb = 1;
@@ -301,7 +313,8 @@ int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, cons
   const bool even = (L->m % 2) == 0;
   cudaError_t e = cudaErrorInvalidValue;
   switch (n) {
-#define DD(NN) case NN: e = even ? launch_dedup<NN, true>(p, (int)grid, 32 * wpb, smem, st) : launch_dedup<NN, false>(p, (int)grid, 32 * wpb, smem, st); break;
+#define DD(NN) case NN: e = fast ? (even ? launch_dedup128<NN, true>(p, (int)grid, 32 * wpb, smem, st) : launch_dedup128<NN, false>(p, (int)grid, 32 * wpb, smem, st)) \
+                             : (even ? launch_dedup<NN, true>(p, (int)grid, 32 * wpb, smem, st) : launch_dedup<NN, false>(p, (int)grid, 32 * wpb, smem, st)); break;
     DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
 #undef DD
     default: return SSHOPM_EUNSUPPORTED;

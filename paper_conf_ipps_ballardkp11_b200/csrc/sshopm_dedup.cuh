@@ -123,4 +123,129 @@ __global__ void __launch_bounds__(256) sshopm_dedup_kernel(const DedupParams p) 
   }
 }
 
+
+// ----------------------------------------------------------------------------
+// Fast path for S = 128: lane l owns starts 4l..4l+3 in registers, loaded as
+// float4 (lambda: 1, x: N, converged: one u32), and the next tensor is
+// prefetched while the current one is clustered.  Same rounds as above (round
+// representative = first unassigned converged start in start order).
+template <int N>
+struct DedupRegs {
+  float4 lam;
+  float4 x[N];      // 4 starts x N components, start-major
+  uint32_t conv;    // 4 bytes
+};
+
+template <int N>
+__device__ __forceinline__ void dedup_load(DedupRegs<N>& r, const DedupParams& p, long long v, int lane) {
+  const long long b = v * 128;
+  r.lam = __ldcs(reinterpret_cast<const float4*>(p.lambda + b) + lane);
+#pragma unroll
+  for (int i = 0; i < N; ++i) r.x[i] = __ldcs(reinterpret_cast<const float4*>(p.x + b * N) + lane * N + i);
+  r.conv = __ldcs(reinterpret_cast<const unsigned int*>(p.conv + b) + lane);
+}
+
+template <int N>
+__device__ __forceinline__ float xcomp(const DedupRegs<N>& r, int c, int j) {   // component j of local start c (c, j compile-time)
+  const int w = c * N + j;
+  const float4 q = r.x[w / 4];
+  return (w % 4 == 0) ? q.x : (w % 4 == 1) ? q.y : (w % 4 == 2) ? q.z : q.w;
+}
+
+template <int N, bool EVEN>
+__global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams p) {
+  constexpr int S = 128, SPL = 4;
+  extern __shared__ float smem[];
+  const int lane = threadIdx.x & 31;
+  const int wib = threadIdx.x >> 5;
+  // per-warp cluster records: lam[S], rep[S], mult[S], x[S][N]
+  float* c_lam = smem + (size_t)wib * S * (N + 3);
+  int* c_rep = reinterpret_cast<int*>(c_lam + S);
+  int* c_mult = c_rep + S;
+  float* c_x = reinterpret_cast<float*>(c_mult + S);
+
+  const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
+  long long v = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
+  DedupRegs<N> nx;
+  if (v < p.n_tensors) dedup_load<N>(nx, p, v, lane);
+  for (; v < p.n_tensors; v += warps) {
+    const DedupRegs<N> cur = nx;
+    if (v + warps < p.n_tensors) dedup_load<N>(nx, p, v + warps, lane);   // prefetch
+    const float lam[SPL] = {cur.lam.x, cur.lam.y, cur.lam.z, cur.lam.w};
+    // cid: -1 unassigned converged, -2 not converged, >= 0 cluster
+    int cid[SPL];
+#pragma unroll
+    for (int c = 0; c < SPL; ++c) cid[c] = ((cur.conv >> (8 * c)) & 0xffu) ? -1 : -2;
+    int ncl = 0;
+    for (;;) {
+      int first = 0x7fffffff;
+#pragma unroll
+      for (int c = SPL - 1; c >= 0; --c)
+        if (cid[c] == -1) first = SPL * lane + c;
+      first = __reduce_min_sync(0xffffffffu, first);
+      if (first == 0x7fffffff) break;
+      const int src = first / SPL, fc = first % SPL;
+      float rl = (fc == 0) ? lam[0] : (fc == 1) ? lam[1] : (fc == 2) ? lam[2] : lam[3];
+      rl = __shfl_sync(0xffffffffu, rl, src);
+      float rx[N];
+      float rn = 0.f;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        float t = (fc == 0) ? xcomp<N>(cur, 0, j) : (fc == 1) ? xcomp<N>(cur, 1, j) : (fc == 2) ? xcomp<N>(cur, 2, j) : xcomp<N>(cur, 3, j);
+        rx[j] = __shfl_sync(0xffffffffu, t, src);
+        rn = fmaf(rx[j], rx[j], rn);
+      }
+      const float ltol = p.lam_tol * fmaxf(1.0f, fabsf(rl));
+      int cnt = 0;
+#pragma unroll
+      for (int c = 0; c < SPL; ++c) {
+        if (cid[c] != -1) continue;
+        bool same = (SPL * lane + c == first);
+        if (!same) {
+          float dot = 0.f, n2 = 0.f;
+#pragma unroll
+          for (int j = 0; j < N; ++j) { const float xv = xcomp<N>(cur, c, j); dot = fmaf(xv, rx[j], dot); n2 = fmaf(xv, xv, n2); }
+          const float lim = p.cos_tol * sqrtf(n2 * rn);
+          if (EVEN) same = fabsf(lam[c] - rl) <= ltol && fabsf(dot) >= lim;
+          else same = (fabsf(lam[c] - rl) <= ltol && dot >= lim) || (fabsf(-lam[c] - rl) <= ltol && -dot >= lim);
+        }
+        if (same) { cid[c] = ncl; ++cnt; }
+      }
+      cnt = __reduce_add_sync(0xffffffffu, cnt);
+      if (lane == 0) {
+        c_lam[ncl] = rl; c_rep[ncl] = first; c_mult[ncl] = cnt;
+#pragma unroll
+        for (int j = 0; j < N; ++j) c_x[ncl * N + j] = rx[j];
+      }
+      ++ncl;
+    }
+    __syncwarp();
+    if (lane == 0) p.out_count[v] = ncl;
+    const long long ob = v * p.kmax;
+    for (int c = lane; c < ncl; c += 32) {
+      const float lc = c_lam[c];
+      int rank = 0;
+      for (int d = 0; d < ncl; ++d) {
+        const float ld = c_lam[d];
+        rank += (ld > lc) || (ld == lc && d < c);
+      }
+      if (rank < p.kmax) {
+        p.out_lambda[ob + rank] = lc;
+#pragma unroll
+        for (int j = 0; j < N; ++j) p.out_x[(ob + rank) * N + j] = c_x[c * N + j];
+        p.out_mult[ob + rank] = c_mult[c];
+        if (p.out_rep) p.out_rep[ob + rank] = c_rep[c];
+      }
+    }
+    for (int slot = ncl + lane; slot < p.kmax; slot += 32) {
+      p.out_lambda[ob + slot] = 0.f;
+#pragma unroll
+      for (int j = 0; j < N; ++j) p.out_x[(ob + slot) * N + j] = 0.f;
+      p.out_mult[ob + slot] = 0;
+      if (p.out_rep) p.out_rep[ob + slot] = -1;
+    }
+    __syncwarp();
+  }
+}
+
 }  // namespace sshopm

@@ -188,6 +188,20 @@ def test_dedup_end_to_end_vs_oracle(dev):
     assert np.all(np.abs(cl[same][filled] - ol[same][filled]) <= 1e-4 * np.maximum(1, np.abs(ol[same][filled])))
 
 
+@pytest.mark.parametrize("S", [16, 100, 128, 200])
+def test_dedup_start_counts(dev, S):
+    """Register fast path (S = 128) and shared-memory general path (other S) follow the same rule."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 5000, 300, 0)
+    st = syn.gen_starts(S, n, 2)
+    s = sh.Solver(m, n)
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.0, 1e-6, 100)
+    cnt, cl, cx, mu, rp = (t.cpu().numpy() for t in s.dedup(lam, x, cv, 1e-2, 0.05, 6))
+    oc, ol, ox, om, orp = D.dedup(lam.cpu().numpy(), x.cpu().numpy(), cv.cpu().numpy().astype(bool), m, 1e-2, 0.05, 6)
+    assert np.array_equal(cnt, oc) and np.array_equal(rp, orp) and np.array_equal(mu, om)
+    assert np.array_equal(cl.astype(np.float64), ol) and np.array_equal(cx.astype(np.float64), ox)
+
+
 def test_dedup_odd_m(dev):
     m, n = 3, 3
     ent = syn.gen_uniform_tensors(m, n, 128, 1)
