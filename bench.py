@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--voxels", type=int, default=0, help="override tensors per rank")
     ap.add_argument("--refill", type=int, default=0)
+    ap.add_argument("--schedule", type=int, default=0, help="0 library default, 1 item-per-lane, 2 tensor-per-lane")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-voxels", type=int, default=0)
@@ -218,7 +219,7 @@ def main():
         if count_iters:
             titers.zero_()
         solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
-                     refill_threshold=a.refill, total_iters=titers if count_iters else None)
+                     refill_threshold=a.refill, total_iters=titers if count_iters else None, schedule=a.schedule)
         solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
         if world > 1:
             SH.gather_records(rec, rank, world)
@@ -241,7 +242,7 @@ def main():
             e0, e1, e2 = ev[i]
             e0.record(stream)
             solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
-                         refill_threshold=a.refill)
+                         refill_threshold=a.refill, schedule=a.schedule)
             e1.record(stream)
             solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
             if world > 1:

@@ -112,6 +112,8 @@ typedef struct {
   unsigned long long* d_total_iters; /* optional device counter: += sum of iters over all lanes (atomicAdd) */
   void* d_workspace;               /* optional caller-owned device workspace, 256-byte aligned, >= sshopm_workspace_size */
   size_t workspace_bytes;          /* its size; a too-small or misaligned workspace returns EINVAL */
+  int schedule;                    /* 0 default, 1 = item per lane (warps claim chunks of whole tensors),
+                                      2 = tensor per lane (a lane walks one tensor's starts); results identical */
 } sshopm_solve_opts;
 
 /* sshopm_solve with options (opts may be NULL).  Launches two kernels on

@@ -35,7 +35,7 @@ class SSHOPMError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
                 ("d_total_iters", ctypes.c_void_p), ("d_workspace", ctypes.c_void_p),
-                ("workspace_bytes", ctypes.c_size_t)]
+                ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int)]
 
 
 def lib():
@@ -165,7 +165,7 @@ class Solver:
         return c.value
 
     def solve(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, out=None, refill_threshold=0,
-              ctas_per_sm=0, total_iters=None, stream=None):
+              ctas_per_sm=0, total_iters=None, stream=None, schedule=0):
         """entries [N, U] f32, starts [S, n] f32 (CUDA) -> (lam [N,S], x [N,S,n], iters [N,S] i32, conv [N,S] u8)."""
         torch = _torch()
         N, S = int(entries.shape[0]), int(starts.shape[0])
@@ -181,7 +181,7 @@ class Solver:
         args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
                 _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
         wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
-        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb)
+        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule))
         if total_iters is not None:
             if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:
                 raise TypeError("total_iters must be a 1-element int64 CUDA tensor")

@@ -181,16 +181,23 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
 
   const int shift = alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2);
   const bool wide = (long long)N * S >= (1LL << 31) - (1LL << 20);
+  // schedule: 1 = item per lane (chunks of whole tensors), 2 = tensor per lane
+  int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
+  if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;
   int bps = 0;
-  cudaError_t e = L->occupancy(shift, wide, &bps);
+  cudaError_t e = L->occupancy(shift, wide, schedule, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
   if (bps < 1) bps = 1;
   if (opts && opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
-  const int chunk_tensors = (S >= 256) ? 1 : (256 + S - 1) / S;      // >= 256 items per chunk
+  const int chunk_tensors = (S >= 256) ? 1 : (256 + S - 1) / S;      // schedule 1: >= 256 items per chunk
   const long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
-  if (n_chunks >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
+  if (n_chunks >= (1LL << 32) - (1LL << 20) || N >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
   long long grid = (long long)sms * bps;
-  if (grid * 8 > n_chunks) grid = (n_chunks + 7) / 8;
+  if (schedule == 1) {
+    if (grid * 8 > n_chunks) grid = (n_chunks + 7) / 8;
+  } else {
+    if (grid * 256 > N) grid = (N + 255) / 256;
+  }
   if (grid < 1) grid = 1;
 
   Workspace ws;
@@ -220,7 +227,7 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   p.maxit = maxit;
   int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : L->default_refill;
   p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
-  e = L->solve(p, shift, wide, (int)grid, st);
+  e = L->solve(p, shift, wide, schedule, (int)grid, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
   h->launches.fetch_add(2);
   return release_workspace(&ws, st);

@@ -19,22 +19,24 @@ void class_index(int32_t* out) {
 }
 
 template <int SH, bool W>
-cudaError_t occ1(int* bps) {
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W>, 256, 0);
+cudaError_t occ1(int schedule, int* bps) {
+  return schedule == 2 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_tpl_kernel<M, N, SH, W>, 256, 0)
+                       : cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W>, 256, 0);
 }
-cudaError_t occupancy(int shift, bool wide, int* bps) {
-  if (wide) return shift == 0 ? occ1<0, true>(bps) : shift == 1 ? occ1<1, true>(bps) : occ1<2, true>(bps);
-  return shift == 0 ? occ1<0, false>(bps) : shift == 1 ? occ1<1, false>(bps) : occ1<2, false>(bps);
+cudaError_t occupancy(int shift, bool wide, int schedule, int* bps) {
+  if (wide) return shift == 0 ? occ1<0, true>(schedule, bps) : shift == 1 ? occ1<1, true>(schedule, bps) : occ1<2, true>(schedule, bps);
+  return shift == 0 ? occ1<0, false>(schedule, bps) : shift == 1 ? occ1<1, false>(schedule, bps) : occ1<2, false>(schedule, bps);
 }
 
 template <int SH, bool W>
-cudaError_t solve1(const SolveParams& p, int grid, cudaStream_t st) {
-  sshopm_solve_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
+cudaError_t solve1(const SolveParams& p, int schedule, int grid, cudaStream_t st) {
+  if (schedule == 2) sshopm_solve_tpl_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
+  else sshopm_solve_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
   return cudaGetLastError();
 }
-cudaError_t solve(const SolveParams& p, int shift, bool wide, int grid, cudaStream_t st) {
-  if (wide) return shift == 0 ? solve1<0, true>(p, grid, st) : shift == 1 ? solve1<1, true>(p, grid, st) : solve1<2, true>(p, grid, st);
-  return shift == 0 ? solve1<0, false>(p, grid, st) : shift == 1 ? solve1<1, false>(p, grid, st) : solve1<2, false>(p, grid, st);
+cudaError_t solve(const SolveParams& p, int shift, bool wide, int schedule, int grid, cudaStream_t st) {
+  if (wide) return shift == 0 ? solve1<0, true>(p, schedule, grid, st) : shift == 1 ? solve1<1, true>(p, schedule, grid, st) : solve1<2, true>(p, schedule, grid, st);
+  return shift == 0 ? solve1<0, false>(p, schedule, grid, st) : shift == 1 ? solve1<1, false>(p, schedule, grid, st) : solve1<2, false>(p, schedule, grid, st);
 }
 
 cudaError_t pack(long long n, const float* e, float4* packed, unsigned int* counter, int n_starts, const float* starts,
@@ -50,7 +52,7 @@ cudaError_t apply(long long n_items, const float4* packed, const float* x, float
 
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
-                      Sh::BFORM ? 1 : 0, 10,
+                      Sh::BFORM ? 1 : 0, 10, 1,
                       class_index, occupancy, pack, solve, apply};
 }  // namespace
 

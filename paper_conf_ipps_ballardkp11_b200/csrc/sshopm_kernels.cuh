@@ -453,6 +453,156 @@ sshopm_solve_kernel(const SolveParams p) {
   }
 }
 
+
+// ------------------------------------------- solve kernel, tensor-per-lane --
+// Schedule 2: a lane owns one tensor at a time and
+// walks its S starts in order, so its coefficient registers are loaded once
+// per S items and a refill only writes the finished item and loads the next
+// start vector.  Lanes claim tensors individually (warp-aggregated atomic on
+// the same counter); the per-step arithmetic is identical to schedule 1, so
+// results are bitwise identical.
+template <int M, int N, int SHIFT, bool WIDE>
+__global__ void __launch_bounds__(256, Shape<M, N>::MINB)
+sshopm_solve_tpl_kernel(const SolveParams p) {
+  constexpr int STEPS = SSHOPM_STEPS;
+  using S = Shape<M, N>;
+  using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
+  constexpr int SST4 = round4(N) / 4;
+  constexpr bool XL = X21<M, N>::v;
+
+  const int lane = threadIdx.x & 31;
+  const uint32_t ltmask = lanemask_lt();
+  const uint32_t FULL = 0xffffffffu;
+  const float alpha = (SHIFT == 2) ? -p.alpha : p.alpha;
+  const float tol = p.tol;
+  const int maxit = p.maxit;
+  const uint32_t S_ = (uint32_t)p.S;
+  const Idx NT = (Idx)p.n_tensors;
+
+  bool exhausted = false;
+  Coefs<M, N> cf;
+  float2 xs[S::NX];
+#pragma unroll
+  for (int i = 0; i < S::NX; ++i) xs[i] = f2(0.f, 0.f);
+  float lamp = 0.f, lam = 0.f;
+  int k = 0;
+  bool has = false, stop = true, conv = false;
+  Idx t = 0;                 // current tensor
+  uint32_t s = S_;           // current start (S_ = needs a tensor)
+  unsigned long long it_sum = 0;
+
+  for (;;) {
+    const uint32_t smask = __ballot_sync(FULL, stop);
+    const uint32_t cnt = __popc(smask);
+    if (cnt >= (uint32_t)p.refill_k || smask == FULL) {     // tensors may be exhausted; starts are not
+      if (stop) {
+        if (has) {
+          const Idx item = t * (Idx)S_ + (Idx)s;
+          p.out_lambda[item] = lam;
+          float* ox = p.out_x + (size_t)item * N;
+#pragma unroll
+          for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
+          p.out_iters[item] = k;
+          p.out_conv[item] = conv ? 1 : 0;
+          it_sum += (unsigned long long)k;
+          ++s;
+        }
+        has = false;
+      }
+      // lanes whose tensor is done claim the next tensors (one atomic per warp)
+      const bool need = stop && s >= S_;
+      const uint32_t nmask = __ballot_sync(FULL, need && !exhausted);
+      if (nmask) {
+        unsigned int base = 0;
+        if (lane == __ffs(nmask) - 1) base = atomicAdd(p.counter, (unsigned int)__popc(nmask));
+        base = __shfl_sync(FULL, base, __ffs(nmask) - 1);
+        if (need && !exhausted) {
+          const Idx nt = (Idx)base + (Idx)__popc(nmask & ltmask);
+          if (nt < NT) {
+            t = nt;
+            s = 0;
+            cf.load(p.packed + t * (Idx)(S::PW / 4));
+          }
+        }
+        if ((long long)base + __popc(nmask) >= (long long)p.n_tensors) exhausted = true;
+      }
+      if (stop && s < S_) {                                  // next start of the lane's tensor
+        has = true;
+        float v[4 * SST4];
+#pragma unroll
+        for (int i = 0; i < SST4; ++i) {
+          const float4 q4 = ldg4(p.starts_n + s * SST4 + i);
+          v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
+        }
+#pragma unroll
+        for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
+        if constexpr (XL) xs[1].y = v[1];
+        k = 0;
+        lamp = __int_as_float(0x7fffffff);
+      }
+      if (__ballot_sync(FULL, has) == 0u) break;
+    }
+
+#pragma unroll
+    for (int rep = 0; rep < STEPS; ++rep) {
+      float2 gp[S::NP > 0 ? S::NP : 1];
+      float gs = 0.f;
+      lam = evaluate<M, N>(cf, xs, gp, gs);
+      conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
+      float2 hp[S::NX];
+      static_for<S::NP>([&](auto qq) {
+        constexpr int i = decltype(qq)::value;
+        if constexpr (SHIFT == 0) hp[i] = gp[i];
+        else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
+        else hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
+      });
+      if constexpr (S::ODD) {
+        float h;
+        if constexpr (SHIFT == 0) h = gs;
+        else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
+        else h = fmaf(alpha, xs[S::NX - 1].x, -gs);
+        hp[S::NX - 1] = f2(h, 0.f);
+      }
+      float nn;
+      {
+        float2 q = __fmul2_rn(hp[0], hp[0]);
+        static_for<S::NX - 1>([&](auto qq) {
+          constexpr int i = decltype(qq)::value + 1;
+          if constexpr (S::ODD && i == S::NX - 1) q.x = fmaf(hp[i].x, hp[i].x, q.x);
+          else q = __ffma2_rn(hp[i], hp[i], q);
+        });
+        nn = q.x + q.y;
+      }
+      const bool deg = !(nn >= 1.17549435e-38f);
+      stop = !has || conv || k >= maxit || deg;
+      const float r = rsqrt_ftz(nn);
+      if constexpr (XL) {
+        const float2 n01 = __fmul2_rn(hp[0], bc(r));
+        const float n2 = hp[1].x * r;
+        xs[0].x = stop ? xs[0].x : n01.x;
+        xs[0].y = stop ? xs[0].y : n01.y;
+        xs[1].x = stop ? xs[1].x : n2;
+        xs[1].y = xs[0].y;
+      } else {
+#pragma unroll
+        for (int i = 0; i < S::NX; ++i) {
+          const float2 nx = __fmul2_rn(hp[i], bc(r));
+          xs[i].x = stop ? xs[i].x : nx.x;
+          xs[i].y = stop ? xs[i].y : nx.y;
+        }
+      }
+      lamp = stop ? lamp : lam;
+      k += stop ? 0 : 1;
+    }
+  }
+
+  if (p.total_iters) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) it_sum += __shfl_xor_sync(0xffffffffu, it_sum, o);
+    if (lane == 0) atomicAdd(p.total_iters, it_sum);
+  }
+}
+
 // ------------------------------------------------------------ apply kernel --
 template <int M, int N>
 __global__ void __launch_bounds__(256)

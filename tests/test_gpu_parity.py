@@ -135,7 +135,8 @@ def test_invariance_across_launch_configs(dev):
     st = syn.gen_starts(128, n, 0)
     base = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
     for kw in [dict(refill_threshold=1), dict(refill_threshold=32), dict(ctas_per_sm=1),
-               dict(refill_threshold=5, ctas_per_sm=2), {}]:
+               dict(refill_threshold=5, ctas_per_sm=2), {}, dict(schedule=2), dict(schedule=2, refill_threshold=3),
+               dict(schedule=2, ctas_per_sm=1, refill_threshold=32), dict(schedule=1)]:
         other = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, **kw)
         for a, b in zip(base, other):
             assert np.array_equal(a, b), kw
@@ -233,13 +234,14 @@ def test_run_host_matches_device_path(dev):
     assert out["total_iters"] == int(it.cpu().numpy().sum())
 
 
+@pytest.mark.parametrize("schedule", [1, 2])
 @pytest.mark.parametrize("V,S", [(1, 1), (3, 1), (5, 7), (40, 2), (2, 300)])
-def test_tiny_chunks(dev, V, S):
+def test_tiny_chunks(dev, V, S, schedule):
     """Chunks smaller than a warp's request (S * tensors < 32) must not overrun (regression)."""
     m, n = 4, 3
     ent = syn.gen_voxels(m, n, 77, V, 0)
     st = syn.gen_starts(S, n, 1)
-    gpu = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
+    gpu = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, schedule=schedule)
     _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, gpu), max_sensitive=0.02)
 
 
