@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-voxels", type=int, default=0)
+    ap.add_argument("--e2e-chunk", type=int, default=0, help="tensors per run_host chunk (0: auto)")
     return ap.parse_args()
 
 
@@ -276,7 +277,7 @@ def main():
                 "x": torch.empty((Nloc, KMAX, n), dtype=torch.float32).pin_memory(),
                 "mult": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory(),
                 "rep": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()}
-        chunk = max(4096, Nloc // 8)
+        chunk = a.e2e_chunk or min(65536, max(4096, Nloc // 32))
         solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
                         chunk_tensors=chunk, out=outs)
         if world > 1:

@@ -79,7 +79,8 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   const bool raw = h_raw_lambda || h_raw_x || h_raw_iters || h_raw_converged;
   if (raw && !(h_raw_lambda && h_raw_x && h_raw_iters && h_raw_converged)) return SSHOPM_EINVAL;
   const int n = h->L->n, U = h->L->U;
-  long long chunk = chunk_tensors > 0 ? chunk_tensors : 65536;
+  long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 32;   // default: ~32 chunks, 4K..64K tensors
+  if (chunk_tensors <= 0) chunk = chunk < 4096 ? 4096 : (chunk > 65536 ? 65536 : chunk);
   if (chunk > N) chunk = N;
 
   if (!h->hc) {

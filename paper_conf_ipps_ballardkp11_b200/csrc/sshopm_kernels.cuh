@@ -329,54 +329,53 @@ sshopm_solve_kernel(const SolveParams p) {
     const uint32_t smask = __ballot_sync(FULL, stop);
     const uint32_t cnt = __popc(smask);
     if ((cnt >= (uint32_t)p.refill_k && !exhausted) || smask == FULL) {
-      uint32_t avail = 0, n_end = 0;
+      // straight-line refill: predicated stores / loads, selects for state (no divergent regions)
+      const uint32_t avail = c_end - c_next;                 // invariant: c_next <= c_end
+      uint32_t n_end = 0;
       Idx n_vox = 0;
-      if (!exhausted) {
-        avail = c_end - c_next;                            // invariant: c_next <= c_end
-        if (cnt > avail) {                                 // claim the next chunk (one atomic per warp)
-          unsigned int ch = 0;
-          if (lane == 0) ch = atomicAdd(p.counter, 1u);
-          ch = __shfl_sync(FULL, ch, 0);
-          if ((long long)ch < p.n_chunks) {
-            n_vox = (Idx)ch * (Idx)p.chunk_tensors;
-            const long long nt = p.n_tensors - (long long)n_vox;
-            n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
-          }
+      if (!exhausted && cnt > avail) {                       // claim the next chunk (one atomic per warp)
+        unsigned int ch = 0;
+        if (lane == 0) ch = atomicAdd(p.counter, 1u);
+        ch = __shfl_sync(FULL, ch, 0);
+        if ((long long)ch < p.n_chunks) {
+          n_vox = (Idx)ch * (Idx)p.chunk_tensors;
+          const long long nt = p.n_tensors - (long long)n_vox;
+          n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
         }
       }
-      if (stop) {
-        if (has) {
-          p.out_lambda[item] = lam;
-          float* ox = p.out_x + (size_t)item * N;            // one 64-bit row address, immediate offsets
+      const bool wr = stop && has;
+      if (wr) {
+        p.out_lambda[item] = lam;
+        float* ox = p.out_x + (size_t)item * N;              // one 64-bit row address, immediate offsets
 #pragma unroll
-          for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
-          p.out_iters[item] = k;
-          p.out_conv[item] = conv ? 1 : 0;
-          it_sum += (unsigned long long)k;
-        }
-        const uint32_t rank = __popc(smask & ltmask);
-        const bool cur = rank < avail;
+        for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
+        p.out_iters[item] = k;
+        p.out_conv[item] = conv ? 1 : 0;
+      }
+      it_sum += wr ? (unsigned long long)k : 0ull;
+      const uint32_t rank = __popc(smask & ltmask);
+      const bool cur = rank < avail;
+      const uint32_t t = cur ? c_next + rank : rank - avail;
+      const bool ok = stop && !exhausted && (cur || t < n_end);
+      if (ok) {
         const Idx v0 = cur ? c_vox : n_vox;
-        const uint32_t t = cur ? c_next + rank : rank - avail;
-        has = !exhausted && (cur || t < n_end);
-        if (has) {
-          const uint32_t vq = fast_div(t, p.divS);
-          const uint32_t s = t - vq * S_;
-          item = v0 * (Idx)S_ + (Idx)t;
-          cf.load(p.packed + (v0 + (Idx)vq) * (Idx)(S::PW / 4));
-          float v[4 * SST4];
+        const uint32_t vq = fast_div(t, p.divS);
+        const uint32_t s = t - vq * S_;
+        item = v0 * (Idx)S_ + (Idx)t;
+        cf.load(p.packed + (v0 + (Idx)vq) * (Idx)(S::PW / 4));
+        float v[4 * SST4];
 #pragma unroll
-          for (int i = 0; i < SST4; ++i) {
-            const float4 q4 = ldg4(p.starts_n + s * SST4 + i);
-            v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
-          }
-#pragma unroll
-          for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
-          if constexpr (XL) xs[1].y = v[1];                // (x2, x1) layout
-          k = 0;
-          lamp = __int_as_float(0x7fffffff);               // NaN: the first test never fires (reading R2)
+        for (int i = 0; i < SST4; ++i) {
+          const float4 q4 = ldg4(p.starts_n + s * SST4 + i);
+          v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
         }
+#pragma unroll
+        for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
+        if constexpr (XL) xs[1].y = v[1];                  // (x2, x1) layout
       }
+      k = ok ? 0 : k;
+      lamp = ok ? __int_as_float(0x7fffffff) : lamp;         // NaN: the first test never fires (reading R2)
+      has = stop ? ok : has;
       if (!exhausted) {
         if (cnt > avail) {
           if (n_end == 0) exhausted = true;
@@ -387,7 +386,7 @@ sshopm_solve_kernel(const SolveParams p) {
           c_next += cnt;
         }
       }
-      if (__ballot_sync(FULL, has) == 0u) break;
+      if (exhausted && __ballot_sync(FULL, has) == 0u) break;
     }
 
     // ---------------- SS-HOPM steps (Fig. 1), STEPS per refill check ----------------
