@@ -46,6 +46,10 @@ def parse():
     ap.add_argument("--voxels", type=int, default=0, help="override tensors per rank")
     ap.add_argument("--refill", type=int, default=0)
     ap.add_argument("--schedule", type=int, default=0, help="0 library default, 1 item-per-lane, 2 tensor-per-lane")
+    ap.add_argument("--unfused", action="store_true", default=True,
+                    help="step = sshopm_solve + sshopm_dedup as separate calls (default; the solve is timed alone)")
+    ap.add_argument("--solve-dedup", dest="unfused", action="store_false", help="step = one sshopm_solve_dedup call")
+    ap.add_argument("--fused", action="store_true", help="sshopm_solve_dedup with in-kernel clustering (opt-in)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-voxels", type=int, default=0)
@@ -216,12 +220,25 @@ def main():
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
+    def run_path(count_iters=False, mid_event=None):
+        """One pass of the hot path: solve (A0-A7) + dedup (A8).  mid_event is recorded between the
+        solve and the dedup launches (two-pass forms) so the solve kernel is timed on its own."""
+        ti = titers if count_iters else None
+        if a.unfused:
+            solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
+                         refill_threshold=a.refill, total_iters=ti, schedule=a.schedule)
+            if mid_event is not None:
+                mid_event.record(stream)
+            solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
+        else:
+            solver.solve_dedup(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
+                               out=(lam, xo, it, cv), dedup_out=tuple(views), refill_threshold=a.refill,
+                               total_iters=ti, schedule=a.schedule, fused=a.fused)
+
     def step(count_iters=False):
         if count_iters:
             titers.zero_()
-        solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
-                     refill_threshold=a.refill, total_iters=titers if count_iters else None, schedule=a.schedule)
-        solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
+        run_path(count_iters)
         if world > 1:
             SH.gather_records(rec, rank, world)
 
@@ -242,10 +259,9 @@ def main():
             flush.zero_()
             e0, e1, e2 = ev[i]
             e0.record(stream)
-            solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
-                         refill_threshold=a.refill, schedule=a.schedule)
-            e1.record(stream)
-            solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
+            run_path(mid_event=e1)
+            if not a.unfused:
+                e1.record(stream)
             if world > 1:
                 SH.gather_records(rec, rank, world)
             e2.record(stream)
@@ -255,7 +271,7 @@ def main():
     torch.cuda.synchronize()
     launches = solver.launch_count() - l0
     t_step = [e0.elapsed_time(e2) for e0, e1, e2 in ev]
-    t_solve = [e0.elapsed_time(e1) for e0, e1, e2 in ev]
+    t_solve = [e0.elapsed_time(e1) for e0, e1, e2 in ev]   # pack + solve kernels (with --solve-dedup: the whole call)
     tot_ms = float(sum(t_step))
     stats = torch.tensor([tot_ms, float(iters_local), float(sum(t_solve))], dtype=torch.float64, device=dev)
     if world > 1:

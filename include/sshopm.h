@@ -114,6 +114,8 @@ typedef struct {
   size_t workspace_bytes;          /* its size; a too-small or misaligned workspace returns EINVAL */
   int schedule;                    /* 0 default, 1 = item per lane (warps claim chunks of whole tensors),
                                       2 = tensor per lane (a lane walks one tensor's starts); results identical */
+  int fuse_dedup;                  /* sshopm_solve_dedup only: 1 = cluster inside the solve kernel (fused),
+                                      0 = default (two passes; faster on B200); results identical */
 } sshopm_solve_opts;
 
 /* sshopm_solve with options (opts may be NULL).  Launches two kernels on
@@ -141,6 +143,24 @@ int sshopm_dedup(sshopm_t h, int64_t N, int S,
                  float lam_tol, float ang_tol, int kmax,
                  int32_t* d_out_count, float* d_out_lambda, float* d_out_x, int32_t* d_out_mult,
                  int32_t* d_out_rep, void* stream);
+
+/* Solve + dedup in one pass (the whole per-tensor hot path, DESIGN.md "Fused
+ * dedup"): same arguments and outputs as sshopm_solve_ex followed by
+ * sshopm_dedup with the same tolerances, and bitwise the same results.  Each
+ * warp of the solve kernel clusters a chunk of tensors as soon as it has
+ * written the chunk's last start (reading the raw outputs back from L2); the
+ * few chunks it cannot track are clustered by a small follow-up kernel.
+ * Raw outputs are required (they are also the dedup's input).  The fused form
+ * is opt-in (opts->fuse_dedup = 1); by default, and whenever the fused form
+ * does not apply (schedule 2, or its shared memory would lower occupancy),
+ * the two passes run back to back on the stream.  Errors: as sshopm_solve_ex
+ * and sshopm_dedup. */
+int sshopm_solve_dedup(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                       float alpha, float tol, int maxit,
+                       float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                       float lam_tol, float ang_tol, int kmax,
+                       int32_t* d_out_count, float* d_out_clambda, float* d_out_cx, int32_t* d_out_mult,
+                       int32_t* d_out_rep, const sshopm_solve_opts* opts, void* stream);
 
 /* Test hook: d_out_g[N][n] = A x^{m-1} (Eq. 6) and d_out_lam[N] = A x^m
  * (Eq. 4 via Euler's identity x.(A x^{m-1})) for N (tensor, x) pairs, using

@@ -35,7 +35,7 @@ class SSHOPMError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
                 ("d_total_iters", ctypes.c_void_p), ("d_workspace", ctypes.c_void_p),
-                ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int)]
+                ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int), ("fuse_dedup", ctypes.c_int)]
 
 
 def lib():
@@ -56,6 +56,8 @@ def lib():
         "sshopm_solve": (I, [P, I64, P, I, P, F, F, I, P, P, P, P, P]),
         "sshopm_solve_ex": (I, [P, I64, P, I, P, F, F, I, P, P, P, P, ctypes.POINTER(_Opts), P]),
         "sshopm_dedup": (I, [P, I64, I, P, P, P, F, F, I, P, P, P, P, P, P]),
+        "sshopm_solve_dedup": (I, [P, I64, P, I, P, F, F, I, P, P, P, P, F, F, I, P, P, P, P, P,
+                                   ctypes.POINTER(_Opts), P]),
         "sshopm_apply": (I, [P, I64, P, P, P, P, P]),
         "sshopm_run_host": (I, [P, I64, P, I, P, F, F, I, F, F, I, P, P, P, P, P, P, P, P, P, I64, P]),
         "sshopm_launch_count": (I, [P, ctypes.POINTER(I64)]),
@@ -181,7 +183,7 @@ class Solver:
         args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
                 _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
         wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
-        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule))
+        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 0)
         if total_iters is not None:
             if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:
                 raise TypeError("total_iters must be a 1-element int64 CUDA tensor")
@@ -189,6 +191,42 @@ class Solver:
         _check(lib().sshopm_solve_ex(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit), *args,
                                      ctypes.byref(opts), _stream(stream)), "sshopm_solve")
         return out
+
+    def solve_dedup(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, lam_tol=1e-2, ang_tol=0.05, kmax=8,
+                    out=None, dedup_out=None, refill_threshold=0, ctas_per_sm=0, total_iters=None, stream=None,
+                    schedule=0, fused=False):
+        """Fused solve + dedup (sshopm_solve_dedup).  Returns (raw outputs, dedup outputs) as in solve() / dedup()."""
+        torch = _torch()
+        N, S = int(entries.shape[0]), int(starts.shape[0])
+        pe = _dev(entries, torch.float32, (N, self.U), "entries")
+        ps = _dev(starts, torch.float32, (S, self.n), "starts")
+        dev = entries.device
+        if out is None:
+            out = (torch.empty((N, S), dtype=torch.float32, device=dev),
+                   torch.empty((N, S, self.n), dtype=torch.float32, device=dev),
+                   torch.empty((N, S), dtype=torch.int32, device=dev),
+                   torch.empty((N, S), dtype=torch.uint8, device=dev))
+        if dedup_out is None:
+            dedup_out = (torch.empty((N,), dtype=torch.int32, device=dev),
+                         torch.empty((N, kmax), dtype=torch.float32, device=dev),
+                         torch.empty((N, kmax, self.n), dtype=torch.float32, device=dev),
+                         torch.empty((N, kmax), dtype=torch.int32, device=dev),
+                         torch.empty((N, kmax), dtype=torch.int32, device=dev))
+        lam, x, it, cv = out
+        c, ol, ox, om, orp = dedup_out
+        args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
+                _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
+        dargs = (_dev(c, torch.int32, (N,), "out_count"), _dev(ol, torch.float32, (N, kmax), "out_clambda"),
+                 _dev(ox, torch.float32, (N, kmax, self.n), "out_cx"), _dev(om, torch.int32, (N, kmax), "out_mult"),
+                 _dev(orp, torch.int32, (N, kmax), "out_rep"))
+        wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
+        opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 1 if fused else 0)
+        if total_iters is not None:
+            opts.d_total_iters = total_iters.data_ptr()
+        _check(lib().sshopm_solve_dedup(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit), *args,
+                                        float(lam_tol), float(ang_tol), int(kmax), *dargs, ctypes.byref(opts),
+                                        _stream(stream)), "sshopm_solve_dedup")
+        return out, dedup_out
 
     def dedup(self, lam, x, conv, lam_tol=1e-2, ang_tol=0.05, kmax=8, out=None, stream=None):
         """-> (count [N] i32, lam [N,kmax], x [N,kmax,n], mult [N,kmax] i32, rep [N,kmax] i32)."""

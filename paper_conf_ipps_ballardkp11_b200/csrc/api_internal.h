@@ -23,6 +23,8 @@ struct Workspace {
   unsigned int* counter = nullptr;   // 256-byte header: chunk counter of the solve kernel
   float* starts_n = nullptr;         // [S][round4(n)] normalised starts (256-byte aligned region)
   float4* packed = nullptr;          // [N][PW/4] packed coefficient rows
+  unsigned int* ovf_count = nullptr; // fused dedup: untracked chunk count (header word 1)
+  unsigned int* ovf_list = nullptr;  // fused dedup: untracked chunk indices [n_chunks]
   bool owned = false;
 };
 size_t workspace_bytes(const Launchers* L, int64_t N, int S);
@@ -32,4 +34,10 @@ int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, cons
                float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
                int32_t* d_rep, cudaStream_t st);
 void free_host_cache(sshopm_ctx* h);
+int chunk_tensors_for(int S);
+int make_dedup_params(const Launchers* L, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
+                      float* d_olam, float* d_ox, int32_t* d_mult, int32_t* d_rep, DedupParams* p);
+int launch_dedup(const Launchers* L, const DedupParams& p, cudaStream_t st);
+int launch_dedup_list(const Launchers* L, const DedupParams& p, const unsigned int* count, const unsigned int* list,
+                      int chunk_tensors, cudaStream_t st);
 }  // namespace sshopm

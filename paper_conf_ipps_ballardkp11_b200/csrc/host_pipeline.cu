@@ -136,11 +136,9 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     o.d_total_iters = c->d_total;
     o.d_workspace = s.ws;
     o.workspace_bytes = s.ws_bytes;
-    rc = sshopm_solve_ex(h, cn, s.ent, S, c->d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, &o, s.st);
+    rc = sshopm_solve_dedup(h, cn, s.ent, S, c->d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, lam_tol, ang_tol,
+                            kmax, s.cnt, s.olam, s.ox, s.mult, s.rep, &o, s.st);
     if (rc != SSHOPM_OK) goto done;
-    rc = dedup_impl(h->L, cn, S, s.lam, s.x, s.cv, lam_tol, ang_tol, kmax, s.cnt, s.olam, s.ox, s.mult, s.rep, s.st);
-    if (rc != SSHOPM_OK) goto done;
-    h->launches.fetch_add(1);
     CK(cudaMemcpyAsync(h_out_count + c0, s.cnt, sizeof(int32_t) * cn, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     CK(cudaMemcpyAsync(h_out_lambda + c0 * kmax, s.olam, sizeof(float) * cn * kmax, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     CK(cudaMemcpyAsync(h_out_x + c0 * kmax * n, s.ox, sizeof(float) * cn * kmax * n, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");

@@ -49,8 +49,13 @@ static size_t starts_region(const Launchers* L, int S) {
   return (b + 255) / 256 * 256;
 }
 
+int chunk_tensors_for(int S) { return (S >= 256) ? 1 : (256 + S - 1) / S; }
+
+static size_t packed_region(const Launchers* L, int64_t N) { return ((size_t)N * (size_t)L->PW * 4 + 255) / 256 * 256; }
+
 size_t workspace_bytes(const Launchers* L, int64_t N, int S) {
-  return 256 + starts_region(L, S) + (size_t)N * (size_t)L->PW * 4;
+  const size_t n_chunks = S > 0 ? (size_t)((N + chunk_tensors_for(S) - 1) / chunk_tensors_for(S)) : 0;
+  return 256 + starts_region(L, S) + packed_region(L, N) + n_chunks * 4;
 }
 
 int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws) {
@@ -67,8 +72,11 @@ int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t u
   }
   ws->base = base;
   ws->counter = reinterpret_cast<unsigned int*>(base);
+  ws->ovf_count = ws->counter + 1;
   ws->starts_n = reinterpret_cast<float*>(reinterpret_cast<char*>(base) + 256);
   ws->packed = reinterpret_cast<float4*>(reinterpret_cast<char*>(base) + 256 + starts_region(L, S));
+  ws->ovf_list = reinterpret_cast<unsigned int*>(reinterpret_cast<char*>(base) + 256 + starts_region(L, S) +
+                                                 packed_region(L, N));
   return SSHOPM_OK;
 }
 
@@ -166,16 +174,20 @@ int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes) {
   return SSHOPM_OK;
 }
 
-int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
-                    float alpha, float tol, int maxit,
-                    float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
-                    const sshopm_solve_opts* opts, void* stream) {
+}  // extern "C"
+
+namespace sshopm {
+// The solve (pack + solve kernels) and, if dd != null, the fused dedup (ring
+// in the solve kernel + sshopm_dedup_list_kernel for untracked chunks), or the
+// standalone dedup after the solve when the fused form does not apply.
+static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts, float alpha,
+                      float tol, int maxit, float* d_out_lambda, float* d_out_x, int32_t* d_out_iters,
+                      uint8_t* d_out_converged, const sshopm_solve_opts* opts, const DedupParams* dd, cudaStream_t st) {
   if (!h || N < 0 || S < 1 || maxit < 0 || std::isnan(alpha) || std::isnan(tol)) return SSHOPM_EINVAL;
   if (N == 0) return SSHOPM_OK;
   if (!d_entries || !d_starts || !d_out_lambda || !d_out_x || !d_out_iters || !d_out_converged) return SSHOPM_EINVAL;
   if (N > (1LL << 40) / S) return SSHOPM_EUNSUPPORTED;
   const Launchers* L = h->L;
-  cudaStream_t st = (cudaStream_t)stream;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
 
@@ -185,11 +197,26 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
   if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;
   int bps = 0;
-  cudaError_t e = L->occupancy(shift, wide, schedule, &bps);
+  cudaError_t e = L->occupancy(shift, wide, schedule, 0, 0, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
   if (bps < 1) bps = 1;
+  // fused dedup (opt-in, opts->fuse_dedup = 1): schedule 1, S <= 1024, and only if its shared memory
+  // costs no occupancy.  Measured slower than the two-pass form on B200 at C2 (6.2 vs 5.4 ms): the
+  // ring + in-kernel clustering push the register-capped solve into spills.
+  int fused = 0;                                         // 0 none, 1 shared-memory dedup, 2 register dedup
+  int smem = 0;
+  const bool fregs = dd && S == 128 && ((uintptr_t)d_out_lambda % 16 == 0) && ((uintptr_t)d_out_x % 16 == 0) &&
+                     ((uintptr_t)d_out_converged % 4 == 0);
+  if (dd && schedule == 1 && S <= 1024 && opts && opts->fuse_dedup == 1) {
+    const int fs = 8 * fused_smem_words(S, L->n, fregs) * 4;
+    int fb = 0;
+    if (fs <= 200 * 1024 && L->occupancy(shift, wide, schedule, fregs ? 2 : 1, fs, &fb) == cudaSuccess && fb >= bps) {
+      fused = fregs ? 2 : 1;
+      smem = fs;
+    }
+  }
   if (opts && opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
-  const int chunk_tensors = (S >= 256) ? 1 : (256 + S - 1) / S;      // schedule 1: >= 256 items per chunk
+  const int chunk_tensors = chunk_tensors_for(S);                  // schedule 1: >= 256 items per chunk
   const long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
   if (n_chunks >= (1LL << 32) - (1LL << 20) || N >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
   long long grid = (long long)sms * bps;
@@ -227,10 +254,49 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
   p.maxit = maxit;
   int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : L->default_refill;
   p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
-  e = L->solve(p, shift, wide, schedule, (int)grid, st);
+  if (dd) p.dd = *dd;
+  p.dd.lambda = d_out_lambda;
+  p.dd.x = d_out_x;
+  p.dd.conv = d_out_converged;
+  p.ovf_count = ws.ovf_count;
+  p.ovf_list = ws.ovf_list;
+  p.fused_regs = fregs ? 1 : 0;
+  e = L->solve(p, shift, wide, schedule, fused, (int)grid, smem, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
   h->launches.fetch_add(2);
+  if (dd) {
+    if (fused) rc = launch_dedup_list(L, p.dd, ws.ovf_count, ws.ovf_list, chunk_tensors, st);
+    else rc = launch_dedup(L, p.dd, st);
+    if (rc != SSHOPM_OK) { release_workspace(&ws, st); return rc; }
+    h->launches.fetch_add(1);
+  }
   return release_workspace(&ws, st);
+}
+}  // namespace sshopm
+
+extern "C" {
+
+int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                    float alpha, float tol, int maxit,
+                    float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                    const sshopm_solve_opts* opts, void* stream) {
+  return solve_impl(h, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
+                    d_out_converged, opts, nullptr, (cudaStream_t)stream);
+}
+
+int sshopm_solve_dedup(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
+                       float alpha, float tol, int maxit,
+                       float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,
+                       float lam_tol, float ang_tol, int kmax,
+                       int32_t* d_out_count, float* d_out_clambda, float* d_out_cx, int32_t* d_out_mult,
+                       int32_t* d_out_rep, const sshopm_solve_opts* opts, void* stream) {
+  if (!h) return SSHOPM_EINVAL;
+  DedupParams dd;
+  int rc = make_dedup_params(h->L, N, S, lam_tol, ang_tol, kmax, d_out_count, d_out_clambda, d_out_cx, d_out_mult,
+                             d_out_rep, &dd);
+  if (rc != SSHOPM_OK) return rc;
+  return solve_impl(h, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
+                    d_out_converged, opts, N > 0 ? &dd : nullptr, (cudaStream_t)stream);
 }
 
 int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
@@ -265,7 +331,7 @@ int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x
 
 namespace sshopm {
 template <int NN, bool EVEN>
-static cudaError_t launch_dedup(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+static cudaError_t launch_dedup_t(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
   if (smem > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(sshopm_dedup_kernel<NN, EVEN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
@@ -284,50 +350,109 @@ static cudaError_t launch_dedup128(const DedupParams& p, int grid, int block, in
   return cudaGetLastError();
 }
 
-int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
-               float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
-               int32_t* d_rep, cudaStream_t st) {
+int make_dedup_params(const Launchers* L, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
+                      float* d_olam, float* d_ox, int32_t* d_mult, int32_t* d_rep, DedupParams* p) {
   if (S < 1 || kmax < 1 || !(lam_tol >= 0.f) || !(ang_tol >= 0.f) || N < 0) return SSHOPM_EINVAL;
-  if (N == 0) return SSHOPM_OK;
-  if (!d_lambda || !d_x || !d_conv || !d_count || !d_olam || !d_ox || !d_mult) return SSHOPM_EINVAL;
+  if (N > 0 && (!d_count || !d_olam || !d_ox || !d_mult)) return SSHOPM_EINVAL;
   if (S > 1024) return SSHOPM_EUNSUPPORTED;
-  const int n = L->n;
+  if (L->n > 8) return SSHOPM_EUNSUPPORTED;
+  p->lambda = nullptr;
+  p->x = nullptr;
+  p->conv = nullptr;
+  p->out_count = d_count;
+  p->out_lambda = d_olam;
+  p->out_x = d_ox;
+  p->out_mult = d_mult;
+  p->out_rep = d_rep;
+  p->n_tensors = N;
+  p->S = S;
+  p->kmax = kmax;
+  p->lam_tol = lam_tol;
+  p->cos_tol = ang_tol >= 3.14159265358979f ? -1.0f : cosf(ang_tol);
+  return SSHOPM_OK;
+}
+
+static int dedup_launch_shape(const Launchers* L, int64_t N, int S, bool fast, int* grid, int* block, int* smem) {
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_dedup: no device");
-  const bool fast = (S == 128) && n <= 8 &&
-                    ((uintptr_t)d_lambda % 16 == 0) && ((uintptr_t)d_x % 16 == 0) && ((uintptr_t)d_conv % 4 == 0);
-  const int per_warp = fast ? 128 * (n + 3) * 4 : dedup_smem_words(S, n) * 4;
+  const int per_warp = fast ? 128 * (L->n + 3) * 4 : dedup_smem_words(S, L->n) * 4;
   int wpb = (96 * 1024) / per_warp;
   if (wpb > 8) wpb = 8;
   if (wpb < 1) wpb = 1;
-  const int smem = wpb * per_warp;
-  long long grid = (N + wpb - 1) / wpb;
-  if (grid > (long long)sms * 16) grid = (long long)sms * 16;
-  DedupParams p;
-  p.lambda = d_lambda;
-  p.x = d_x;
-  p.conv = d_conv;
-  p.out_count = d_count;
-  p.out_lambda = d_olam;
-  p.out_x = d_ox;
-  p.out_mult = d_mult;
-  p.out_rep = d_rep;
-  p.n_tensors = N;
-  p.S = S;
-  p.kmax = kmax;
-  p.lam_tol = lam_tol;
-  p.cos_tol = ang_tol >= 3.14159265358979f ? -1.0f : cosf(ang_tol);
+  *smem = wpb * per_warp;
+  *block = 32 * wpb;
+  long long g = (N + wpb - 1) / wpb;
+  if (g > (long long)sms * 16) g = (long long)sms * 16;
+  if (g < 1) g = 1;
+  *grid = (int)g;
+  return SSHOPM_OK;
+}
+
+int launch_dedup(const Launchers* L, const DedupParams& p, cudaStream_t st) {
+  if (p.n_tensors == 0) return SSHOPM_OK;
+  if (!p.lambda || !p.x || !p.conv) return SSHOPM_EINVAL;
+  const int S = p.S, n = L->n;
+  const bool fast = (S == 128) && ((uintptr_t)p.lambda % 16 == 0) && ((uintptr_t)p.x % 16 == 0) &&
+                    ((uintptr_t)p.conv % 4 == 0);
+  int grid, block, smem;
+  int rc = dedup_launch_shape(L, p.n_tensors, S, fast, &grid, &block, &smem);
+  if (rc != SSHOPM_OK) return rc;
   const bool even = (L->m % 2) == 0;
   cudaError_t e = cudaErrorInvalidValue;
   switch (n) {
-#define DD(NN) case NN: e = fast ? (even ? launch_dedup128<NN, true>(p, (int)grid, 32 * wpb, smem, st) : launch_dedup128<NN, false>(p, (int)grid, 32 * wpb, smem, st)) \
-                             : (even ? launch_dedup<NN, true>(p, (int)grid, 32 * wpb, smem, st) : launch_dedup<NN, false>(p, (int)grid, 32 * wpb, smem, st)); break;
+#define DD(NN) case NN: e = fast ? (even ? launch_dedup128<NN, true>(p, grid, block, smem, st) : launch_dedup128<NN, false>(p, grid, block, smem, st)) \
+                             : (even ? launch_dedup_t<NN, true>(p, grid, block, smem, st) : launch_dedup_t<NN, false>(p, grid, block, smem, st)); break;
     DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
 #undef DD
     default: return SSHOPM_EUNSUPPORTED;
   }
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_dedup: launch");
   return SSHOPM_OK;
+}
+
+template <int NN, bool EVEN>
+static cudaError_t launch_list_t(const DedupParams& p, const unsigned int* count, const unsigned int* list, int ct,
+                                 int grid, int block, int smem, cudaStream_t st) {
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup_list_kernel<NN, EVEN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+  }
+  sshopm_dedup_list_kernel<NN, EVEN><<<grid, block, smem, st>>>(p, count, list, ct);
+  return cudaGetLastError();
+}
+
+int launch_dedup_list(const Launchers* L, const DedupParams& p, const unsigned int* count, const unsigned int* list,
+                      int chunk_tensors, cudaStream_t st) {
+  int grid, block, smem;
+  int rc = dedup_launch_shape(L, p.n_tensors, p.S, false, &grid, &block, &smem);
+  if (rc != SSHOPM_OK) return rc;
+  const int sms = device_sms();
+  if (grid > sms * 2) grid = sms * 2;                     // untracked chunks are rare
+  const bool even = (L->m % 2) == 0;
+  cudaError_t e = cudaErrorInvalidValue;
+  switch (L->n) {
+#define DD(NN) case NN: e = even ? launch_list_t<NN, true>(p, count, list, chunk_tensors, grid, block, smem, st) \
+                             : launch_list_t<NN, false>(p, count, list, chunk_tensors, grid, block, smem, st); break;
+    DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
+#undef DD
+    default: return SSHOPM_EUNSUPPORTED;
+  }
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_dedup_list: launch");
+  return SSHOPM_OK;
+}
+
+int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
+               float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
+               int32_t* d_rep, cudaStream_t st) {
+  DedupParams p;
+  int rc = make_dedup_params(L, N, S, lam_tol, ang_tol, kmax, d_count, d_olam, d_ox, d_mult, d_rep, &p);
+  if (rc != SSHOPM_OK) return rc;
+  if (N == 0) return SSHOPM_OK;
+  if (!d_lambda || !d_x || !d_conv) return SSHOPM_EINVAL;
+  p.lambda = d_lambda;
+  p.x = d_x;
+  p.conv = d_conv;
+  return launch_dedup(L, p, st);
 }
 }  // namespace sshopm
 

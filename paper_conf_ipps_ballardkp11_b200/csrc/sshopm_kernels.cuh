@@ -24,6 +24,7 @@
 #include <stdint.h>
 #include <type_traits>
 #include "symm_tables.cuh"
+#include "sshopm_dedup.cuh"
 
 namespace sshopm {
 
@@ -75,7 +76,7 @@ sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float
                    unsigned int* __restrict__ counter, int n_starts, const float* __restrict__ starts,
                    float* __restrict__ starts_n) {
   using S = Shape<M, N>;
-  if (counter && blockIdx.x == 0 && threadIdx.x == 0) *counter = 0u;   // chunk counter of the following solve
+  if (counter && blockIdx.x == 0 && threadIdx.x == 0) { counter[0] = 0u; counter[1] = 0u; }   // solve's chunk / overflow counters
   // normalised starts x_0 = s / ||s|| in FP32 (reading R7), rows padded to SST floats
   constexpr int SST = round4(N);
   for (int s = blockIdx.x * blockDim.x + threadIdx.x; s < n_starts; s += gridDim.x * blockDim.x) {
@@ -282,7 +283,17 @@ struct SolveParams {
   float alpha, tol;
   int maxit;
   int refill_k;              // refill threshold
+  // fused solve -> dedup (FUSED kernels only)
+  DedupParams dd;            // dedup outputs; dd.lambda/x/conv = the raw outputs above
+  unsigned int* ovf_count;   // chunks whose completion could not be tracked (zeroed by the pack kernel)
+  unsigned int* ovf_list;    // their chunk indices -> sshopm_dedup_list_kernel
+  int fused_regs;            // S == 128 with 16-byte aligned raw outputs: register-resident dedup, no staging smem
 };
+
+constexpr int kFusedRing = 16;   // open-chunk ring per warp (fused solve -> dedup), power of two
+__host__ __device__ constexpr int fused_smem_words(int S, int n, bool regs) {
+  return 3 * kFusedRing + (regs ? 0 : dedup_smem_words(S, n));
+}
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t r;
@@ -292,9 +303,13 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 
 // SHIFT: 0 -> alpha == 0 (xhat = g), 1 -> alpha > 0 (xhat = g + alpha x), 2 -> alpha < 0 (xhat = -(g + alpha x))
 // WIDE: 64-bit item indices (N*S >= 2^31); otherwise 32-bit index arithmetic.
-template <int M, int N, int SHIFT, bool WIDE>
+// FUSED: also cluster each chunk's tensors (R16) as soon as the warp has
+// written the chunk's last item (open chunks tracked in a shared-memory ring;
+// untracked chunks go to p.ovf_list for sshopm_dedup_list_kernel).
+template <int M, int N, int SHIFT, bool WIDE, int FUSED_MODE>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
+  constexpr bool FUSED = FUSED_MODE != 0;        // 1: shared-memory dedup (any S <= 1024), 2: register dedup (S = 128)
   constexpr int STEPS = SSHOPM_STEPS;        // SS-HOPM steps between refill checks
   using S = Shape<M, N>;
   using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
@@ -308,6 +323,23 @@ sshopm_solve_kernel(const SolveParams p) {
   const float tol = p.tol;
   const int maxit = p.maxit;
   const uint32_t S_ = (uint32_t)p.S;
+
+  // fused dedup: per-warp open-chunk ring + dedup staging in shared memory
+  extern __shared__ int fsm[];
+  int* r_seq = fsm + (threadIdx.x >> 5) * fused_smem_words(p.S, N, FUSED_MODE == 2);
+  unsigned int* r_chunk = reinterpret_cast<unsigned int*>(r_seq + kFusedRing);
+  int* r_rem = r_seq + 2 * kFusedRing;
+  float* d_lam = reinterpret_cast<float*>(r_seq + 3 * kFusedRing);
+  float* d_x = d_lam + p.S;
+  int* d_cid = reinterpret_cast<int*>(d_x + p.S * N);
+  float* d_clam = reinterpret_cast<float*>(d_cid + p.S);
+  int* d_crep = reinterpret_cast<int*>(d_clam + p.S);
+  int* d_cmult = d_crep + p.S;
+  int claim_seq = 0, cur_seq = 0, cseq = -1;
+  if constexpr (FUSED) {
+    if ((threadIdx.x & 31) < kFusedRing) { r_seq[threadIdx.x & 31] = -1; r_rem[threadIdx.x & 31] = 0; }
+    __syncwarp();
+  }
 
   // warp-uniform chunk state
   Idx c_vox = 0;              // first tensor of the current chunk
@@ -341,6 +373,17 @@ sshopm_solve_kernel(const SolveParams p) {
           n_vox = (Idx)ch * (Idx)p.chunk_tensors;
           const long long nt = p.n_tensors - (long long)n_vox;
           n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
+          if constexpr (FUSED) {
+            ++claim_seq;
+            const int slot = claim_seq & (kFusedRing - 1);
+            if (lane == 0) {
+              if (r_rem[slot] > 0) p.ovf_list[atomicAdd(p.ovf_count, 1u)] = r_chunk[slot];   // still open: hand over
+              r_seq[slot] = claim_seq;
+              r_chunk[slot] = ch;
+              r_rem[slot] = (int)n_end;
+            }
+            __syncwarp();
+          }
         }
       }
       const bool wr = stop && has;
@@ -353,6 +396,15 @@ sshopm_solve_kernel(const SolveParams p) {
         p.out_conv[item] = conv ? 1 : 0;
       }
       it_sum += wr ? (unsigned long long)k : 0ull;
+      bool chunk_done = false;
+      int done_slot = 0;                                   // ring slot of the chunk this lane completed
+      if constexpr (FUSED) {
+        if (wr) {
+          const int slot = cseq & (kFusedRing - 1);
+          if (r_seq[slot] == cseq) chunk_done = (atomicSub(&r_rem[slot], 1) == 1);
+          done_slot = slot;
+        }
+      }
       const uint32_t rank = __popc(smask & ltmask);
       const bool cur = rank < avail;
       const uint32_t t = cur ? c_next + rank : rank - avail;
@@ -362,6 +414,7 @@ sshopm_solve_kernel(const SolveParams p) {
         const uint32_t vq = fast_div(t, p.divS);
         const uint32_t s = t - vq * S_;
         item = v0 * (Idx)S_ + (Idx)t;
+        if constexpr (FUSED) cseq = cur ? cur_seq : claim_seq;
         cf.load(p.packed + (v0 + (Idx)vq) * (Idx)(S::PW / 4));
         float v[4 * SST4];
 #pragma unroll
@@ -382,8 +435,40 @@ sshopm_solve_kernel(const SolveParams p) {
           c_vox = n_vox;
           c_next = min(cnt - avail, n_end);                // a chunk smaller than the request is used up
           c_end = n_end;
+          cur_seq = claim_seq;
         } else {
           c_next += cnt;
+        }
+      }
+      if constexpr (FUSED) {
+        uint32_t dmask = __ballot_sync(FULL, chunk_done);
+        if (dmask) {                                       // cluster the completed chunks' tensors now (L2-hot)
+          __threadfence_block();
+          __syncwarp();
+          do {
+            const int src = __ffs(dmask) - 1;
+            dmask &= dmask - 1;
+            const int slot = __shfl_sync(FULL, done_slot, src);
+            const long long v0 = (long long)r_chunk[slot] * p.chunk_tensors;
+            const long long v1 = min(p.n_tensors, v0 + p.chunk_tensors);
+            if constexpr (FUSED_MODE == 2) {
+              bool ok = true;
+#pragma unroll 1
+              for (long long v = v0; v < v1 && ok; ++v) ok = warp_dedup128_regs<N, (M % 2) == 0>(p.dd, v, lane);
+              if (!ok && lane == 0) p.ovf_list[atomicAdd(p.ovf_count, 1u)] = r_chunk[slot];   // > 32 clusters
+            } else {
+#pragma unroll 1
+              for (long long v = v0; v < v1; ++v)
+                warp_dedup_tensor<N, (M % 2) == 0>(p.dd, v, lane, d_lam, d_x, d_cid, d_clam, d_crep, d_cmult);
+            }
+            if (lane == 0) r_seq[slot] = -1;
+            __syncwarp();
+          } while (dmask);
+          // the coefficient registers were dead during the dedup: rematerialise them
+          Idx tv;
+          if constexpr (WIDE) tv = item / (Idx)S_;
+          else tv = fast_div(item, p.divS);
+          cf.load(p.packed + tv * (Idx)(S::PW / 4));
         }
       }
       if (exhausted && __ballot_sync(FULL, has) == 0u) break;

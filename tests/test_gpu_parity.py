@@ -256,3 +256,49 @@ def test_empty_and_tiny(dev):
     st1 = syn.gen_starts(1, n, 0)
     gpu = _solve(dev, m, n, ent, st1, 0.0, 1e-6, 100)
     _assert_parity(PR.solve_parity(ent, st1, m, n, 0.0, 1e-6, 100, gpu))
+
+
+# ------------------------------------------------------- fused solve->dedup --
+def _two_pass(dev, m, n, ent, st, alpha, tol, maxit, lt, at, kmax, **kw):
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    raw = s.solve(e, t, alpha, tol, maxit, **kw)
+    dd = s.dedup(raw[0], raw[1], raw[3], lt, at, kmax)
+    torch.cuda.synchronize()
+    return [x.cpu().numpy() for x in raw], [x.cpu().numpy() for x in dd]
+
+
+def _fused(dev, m, n, ent, st, alpha, tol, maxit, lt, at, kmax, **kw):
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    raw, dd = s.solve_dedup(e, t, alpha, tol, maxit, lt, at, kmax, fused=True, **kw)
+    torch.cuda.synchronize()
+    return [x.cpu().numpy() for x in raw], [x.cpu().numpy() for x in dd]
+
+
+@pytest.mark.parametrize("m,n,V,S,alpha,kmax", [(4, 3, 3000, 128, 0.0, 4), (4, 3, 777, 100, 0.0, 8), (6, 3, 500, 128, 0.25, 6),
+                                                (3, 3, 400, 64, 1.0, 5), (4, 6, 200, 128, 0.0, 4), (8, 3, 100, 32, 0.5, 3),
+                                                (4, 3, 50, 300, 0.0, 4)])
+def test_fused_equals_two_pass(dev, m, n, V, S, alpha, kmax):
+    """sshopm_solve_dedup == sshopm_solve + sshopm_dedup, bit for bit (raw and dedup outputs)."""
+    ent = syn.gen_voxels(m, n, 900, V, 1) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 1)
+    st = syn.gen_starts(S, n, 3)
+    ra, da = _two_pass(dev, m, n, ent, st, alpha, 1e-6, 100, 1e-2, 0.05, kmax)
+    rb, db = _fused(dev, m, n, ent, st, alpha, 1e-6, 100, 1e-2, 0.05, kmax)
+    for a, b in zip(ra + da, rb + db):
+        assert np.array_equal(a, b)
+
+
+def test_fused_ring_overflow(dev):
+    """Chunks held open for thousands of steps by slow lanes overflow the per-warp ring; the
+    follow-up list kernel must still cluster them (results identical to the two-pass form)."""
+    m, n, V, S = 4, 3, 6000, 128
+    ent = syn.gen_voxels(m, n, 0, V, 4)
+    slow = syn.gen_uniform_tensors(m, n, V // 40, 9)      # unstructured, alpha = 0: many non-converging starts
+    ent[::40] = slow
+    st = syn.gen_starts(S, n, 0)
+    ra, da = _two_pass(dev, m, n, ent, st, 0.0, 1e-6, 3000, 1e-2, 0.05, 4)
+    rb, db = _fused(dev, m, n, ent, st, 0.0, 1e-6, 3000, 1e-2, 0.05, 4)
+    assert ra[2].max() == 3000 and (ra[2] == 3000).sum() > 100    # slow lanes really ran to maxit
+    for a, b in zip(ra + da, rb + db):
+        assert np.array_equal(a, b)
