@@ -116,6 +116,12 @@ typedef struct {
                                       2 = tensor per lane (a lane walks one tensor's starts); results identical */
   int fuse_dedup;                  /* sshopm_solve_dedup only: 1 = cluster inside the solve kernel (fused),
                                       0 = default (two passes; faster on B200); results identical */
+  int alpha_mode;                  /* shift: 0 = the scalar alpha argument (default);
+                                      1 = per tensor, d_alpha[N] (device); 2 = per tensor automatic convex shift
+                                      alpha_t = +(m-1) sum_{all indices} |a| (>= beta(A): lambda_k nondecreasing,
+                                      converges to local maxima, Kolda-Mayo [1]); 3 = automatic concave shift -(...)
+                                      (minima).  Modes 1-3 use schedule 1. */
+  const float* d_alpha;            /* alpha_mode 1: per-tensor shifts [N] */
 } sshopm_solve_opts;
 
 /* sshopm_solve with options (opts may be NULL).  Launches two kernels on

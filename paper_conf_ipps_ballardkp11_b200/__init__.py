@@ -35,7 +35,10 @@ class SSHOPMError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
                 ("d_total_iters", ctypes.c_void_p), ("d_workspace", ctypes.c_void_p),
-                ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int), ("fuse_dedup", ctypes.c_int)]
+                ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int), ("fuse_dedup", ctypes.c_int),
+                ("alpha_mode", ctypes.c_int), ("d_alpha", ctypes.c_void_p)]
+
+ALPHA_MODES = {"scalar": 0, "per_tensor": 1, "auto_max": 2, "auto_min": 3}
 
 
 def lib():
@@ -161,6 +164,22 @@ class Solver:
         base = ws.data_ptr()
         return ctypes.c_void_p((base + 255) // 256 * 256), need
 
+    @staticmethod
+    def _alpha_opts(alpha, N, opts):
+        """alpha: float (scalar shift), a CUDA float32 tensor [N] (per tensor), or 'auto_max' / 'auto_min'."""
+        if isinstance(alpha, str):
+            if alpha not in ("auto_max", "auto_min"):
+                raise ValueError("alpha must be a float, a [N] tensor, 'auto_max' or 'auto_min'")
+            opts.alpha_mode = ALPHA_MODES[alpha]
+            return 0.0
+        if hasattr(alpha, "data_ptr"):
+            torch = _torch()
+            _dev(alpha, torch.float32, (N,), "alpha")
+            opts.alpha_mode = 1
+            opts.d_alpha = alpha.data_ptr()
+            return 0.0
+        return float(alpha)
+
     def launch_count(self):
         c = ctypes.c_int64()
         _check(lib().sshopm_launch_count(self._h, ctypes.byref(c)), "sshopm_launch_count")
@@ -184,6 +203,7 @@ class Solver:
                 _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
         wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
         opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 0)
+        alpha = self._alpha_opts(alpha, N, opts)
         if total_iters is not None:
             if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:
                 raise TypeError("total_iters must be a 1-element int64 CUDA tensor")
@@ -221,6 +241,7 @@ class Solver:
                  _dev(orp, torch.int32, (N, kmax), "out_rep"))
         wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
         opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 1 if fused else 0)
+        alpha = self._alpha_opts(alpha, N, opts)
         if total_iters is not None:
             opts.d_total_iters = total_iters.data_ptr()
         _check(lib().sshopm_solve_dedup(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit), *args,

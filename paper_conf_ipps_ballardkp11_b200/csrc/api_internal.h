@@ -25,6 +25,7 @@ struct Workspace {
   float4* packed = nullptr;          // [N][PW/4] packed coefficient rows
   unsigned int* ovf_count = nullptr; // fused dedup: untracked chunk count (header word 1)
   unsigned int* ovf_list = nullptr;  // fused dedup: untracked chunk indices [n_chunks]
+  float* alpha_t = nullptr;          // per-tensor shift [N] (alpha modes 1-3)
   bool owned = false;
 };
 size_t workspace_bytes(const Launchers* L, int64_t N, int S);

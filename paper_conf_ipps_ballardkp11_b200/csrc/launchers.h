@@ -15,7 +15,8 @@ struct Launchers {
   void (*class_index)(int32_t* out);   // [U][m], 0-based
   cudaError_t (*occupancy)(int shift, bool wide, int schedule, int fused, int smem_bytes, int* blocks_per_sm);
   cudaError_t (*pack)(long long n_tensors, const float* entries, float4* packed, unsigned int* counter, int n_starts,
-                      const float* starts, float* starts_n, int grid, cudaStream_t st);
+                      const float* starts, float* starts_n, int alpha_mode, const float* alpha_in, float* alpha_t,
+                      int grid, cudaStream_t st);
   cudaError_t (*solve)(const SolveParams& p, int shift, bool wide, int schedule, int fused, int grid, int smem_bytes,
                        cudaStream_t st);
   cudaError_t (*apply)(long long n_items, const float4* packed, const float* x, float* g, float* lam, int grid,

@@ -53,9 +53,13 @@ int chunk_tensors_for(int S) { return (S >= 256) ? 1 : (256 + S - 1) / S; }
 
 static size_t packed_region(const Launchers* L, int64_t N) { return ((size_t)N * (size_t)L->PW * 4 + 255) / 256 * 256; }
 
-size_t workspace_bytes(const Launchers* L, int64_t N, int S) {
+static size_t chunk_list_region(int64_t N, int S) {
   const size_t n_chunks = S > 0 ? (size_t)((N + chunk_tensors_for(S) - 1) / chunk_tensors_for(S)) : 0;
-  return 256 + starts_region(L, S) + packed_region(L, N) + n_chunks * 4;
+  return (n_chunks * 4 + 255) / 256 * 256;
+}
+
+size_t workspace_bytes(const Launchers* L, int64_t N, int S) {
+  return 256 + starts_region(L, S) + packed_region(L, N) + chunk_list_region(N, S) + (size_t)N * 4;
 }
 
 int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws) {
@@ -77,6 +81,8 @@ int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t u
   ws->packed = reinterpret_cast<float4*>(reinterpret_cast<char*>(base) + 256 + starts_region(L, S));
   ws->ovf_list = reinterpret_cast<unsigned int*>(reinterpret_cast<char*>(base) + 256 + starts_region(L, S) +
                                                  packed_region(L, N));
+  ws->alpha_t = reinterpret_cast<float*>(reinterpret_cast<char*>(base) + 256 + starts_region(L, S) + packed_region(L, N) +
+                                         chunk_list_region(N, S));
   return SSHOPM_OK;
 }
 
@@ -191,11 +197,16 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
 
-  const int shift = alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2);
+  // shift: scalar alpha (R4), or per tensor (alpha_mode 1: caller's array; 2 / 3: +- convexity bound, R17)
+  const int alpha_mode = opts ? opts->alpha_mode : 0;
+  if (alpha_mode < 0 || alpha_mode > 3) return SSHOPM_EINVAL;
+  if (alpha_mode == 1 && !opts->d_alpha) return SSHOPM_EINVAL;
+  const int shift = alpha_mode ? 3 : (alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2));
   const bool wide = (long long)N * S >= (1LL << 31) - (1LL << 20);
   // schedule: 1 = item per lane (chunks of whole tensors), 2 = tensor per lane
   int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
   if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;
+  if (shift == 3) schedule = 1;                                  // per-tensor alpha: schedule 1 only
   int bps = 0;
   cudaError_t e = L->occupancy(shift, wide, schedule, 0, 0, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
@@ -232,7 +243,8 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   if (rc != SSHOPM_OK) return rc;
   long long pgrid = ((N > S ? N : S) + 255) / 256;
   if (pgrid > (long long)sms * 8) pgrid = (long long)sms * 8;
-  e = L->pack(N, d_entries, ws.packed, ws.counter, S, d_starts, ws.starts_n, (int)pgrid, st);
+  e = L->pack(N, d_entries, ws.packed, ws.counter, S, d_starts, ws.starts_n, alpha_mode,
+              alpha_mode == 1 ? opts->d_alpha : nullptr, ws.alpha_t, (int)pgrid, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: pack launch"); }
 
   SolveParams p;
@@ -250,6 +262,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   p.S = S;
   p.divS = make_fastdiv((uint32_t)S);
   p.alpha = alpha;
+  p.alpha_t = ws.alpha_t;
   p.tol = tol;
   p.maxit = maxit;
   int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : L->default_refill;
@@ -320,7 +333,7 @@ int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x
   Workspace ws;
   int rc = acquire_workspace(h->L, N, 0, nullptr, 0, st, &ws);
   if (rc != SSHOPM_OK) return rc;
-  cudaError_t e = h->L->pack(N, d_entries, ws.packed, nullptr, 0, nullptr, nullptr, (int)grid, st);
+  cudaError_t e = h->L->pack(N, d_entries, ws.packed, nullptr, 0, nullptr, nullptr, 0, nullptr, nullptr, (int)grid, st);
   if (e == cudaSuccess) e = h->L->apply(N, ws.packed, d_x, d_out_g, d_out_lam, (int)grid, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_apply: launch"); }
   h->launches.fetch_add(2);

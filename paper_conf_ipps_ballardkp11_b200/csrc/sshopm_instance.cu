@@ -20,23 +20,36 @@ void class_index(int32_t* out) {
 
 template <int SH, bool W, int F>
 cudaError_t occ2(int schedule, int smem, int* bps) {
-  return schedule == 2 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_tpl_kernel<M, N, SH, W>, 256, 0)
-                       : cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W, F>, 256, smem);
+  if constexpr (SH == 3) {
+    if (schedule == 2) return cudaErrorInvalidValue;         // per-tensor alpha: schedule 1 only
+  } else {
+    if (schedule == 2) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_tpl_kernel<M, N, SH, W>, 256, 0);
+  }
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W, F>, 256, smem);
 }
 template <int SH, bool W>
 cudaError_t occ1(int schedule, int fused, int smem, int* bps) {
   return fused == 2 ? occ2<SH, W, 2>(schedule, smem, bps) : fused == 1 ? occ2<SH, W, 1>(schedule, smem, bps)
                     : occ2<SH, W, 0>(schedule, smem, bps);
 }
+template <bool W>
+cudaError_t occw(int shift, int schedule, int fused, int smem, int* bps) {
+  switch (shift) {
+    case 0: return occ1<0, W>(schedule, fused, smem, bps);
+    case 1: return occ1<1, W>(schedule, fused, smem, bps);
+    case 2: return occ1<2, W>(schedule, fused, smem, bps);
+    default: return occ1<3, W>(schedule, fused, smem, bps);
+  }
+}
 cudaError_t occupancy(int shift, bool wide, int schedule, int fused, int smem, int* bps) {
-  if (wide) return shift == 0 ? occ1<0, true>(schedule, fused, smem, bps) : shift == 1 ? occ1<1, true>(schedule, fused, smem, bps) : occ1<2, true>(schedule, fused, smem, bps);
-  return shift == 0 ? occ1<0, false>(schedule, fused, smem, bps) : shift == 1 ? occ1<1, false>(schedule, fused, smem, bps) : occ1<2, false>(schedule, fused, smem, bps);
+  return wide ? occw<true>(shift, schedule, fused, smem, bps) : occw<false>(shift, schedule, fused, smem, bps);
 }
 
 template <int SH, bool W, int F>
 cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaStream_t st) {
   if (schedule == 2) {
-    sshopm_solve_tpl_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
+    if constexpr (SH == 3) return cudaErrorInvalidValue;     // per-tensor alpha: schedule 1 only
+    else sshopm_solve_tpl_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
   } else {
     if (smem > 48 * 1024) {
       cudaError_t e = cudaFuncSetAttribute(sshopm_solve_kernel<M, N, SH, W, F>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -51,14 +64,23 @@ cudaError_t solve1(const SolveParams& p, int schedule, int fused, int grid, int 
   return fused == 2 ? solve2<SH, W, 2>(p, schedule, grid, smem, st) : fused == 1 ? solve2<SH, W, 1>(p, schedule, grid, smem, st)
                     : solve2<SH, W, 0>(p, schedule, grid, smem, st);
 }
+template <bool W>
+cudaError_t solvew(const SolveParams& p, int shift, int schedule, int fused, int grid, int smem, cudaStream_t st) {
+  switch (shift) {
+    case 0: return solve1<0, W>(p, schedule, fused, grid, smem, st);
+    case 1: return solve1<1, W>(p, schedule, fused, grid, smem, st);
+    case 2: return solve1<2, W>(p, schedule, fused, grid, smem, st);
+    default: return solve1<3, W>(p, schedule, fused, grid, smem, st);
+  }
+}
 cudaError_t solve(const SolveParams& p, int shift, bool wide, int schedule, int fused, int grid, int smem, cudaStream_t st) {
-  if (wide) return shift == 0 ? solve1<0, true>(p, schedule, fused, grid, smem, st) : shift == 1 ? solve1<1, true>(p, schedule, fused, grid, smem, st) : solve1<2, true>(p, schedule, fused, grid, smem, st);
-  return shift == 0 ? solve1<0, false>(p, schedule, fused, grid, smem, st) : shift == 1 ? solve1<1, false>(p, schedule, fused, grid, smem, st) : solve1<2, false>(p, schedule, fused, grid, smem, st);
+  return wide ? solvew<true>(p, shift, schedule, fused, grid, smem, st) : solvew<false>(p, shift, schedule, fused, grid, smem, st);
 }
 
 cudaError_t pack(long long n, const float* e, float4* packed, unsigned int* counter, int n_starts, const float* starts,
-                 float* starts_n, int grid, cudaStream_t st) {
-  sshopm_pack_kernel<M, N><<<grid, 256, 0, st>>>(n, e, packed, counter, n_starts, starts, starts_n);
+                 float* starts_n, int alpha_mode, const float* alpha_in, float* alpha_t, int grid, cudaStream_t st) {
+  sshopm_pack_kernel<M, N><<<grid, 256, 0, st>>>(n, e, packed, counter, n_starts, starts, starts_n, alpha_mode, alpha_in,
+                                                 alpha_t);
   return cudaGetLastError();
 }
 

@@ -74,7 +74,8 @@ template <int M, int N>
 __global__ void __launch_bounds__(256)
 sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float4* __restrict__ packed,
                    unsigned int* __restrict__ counter, int n_starts, const float* __restrict__ starts,
-                   float* __restrict__ starts_n) {
+                   float* __restrict__ starts_n, int alpha_mode, const float* __restrict__ alpha_in,
+                   float* __restrict__ alpha_t) {
   using S = Shape<M, N>;
   if (counter && blockIdx.x == 0 && threadIdx.x == 0) { counter[0] = 0u; counter[1] = 0u; }   // solve's chunk / overflow counters
   // normalised starts x_0 = s / ||s|| in FP32 (reading R7), rows padded to SST floats
@@ -113,6 +114,19 @@ sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float
     } else {
 #pragma unroll
       for (int c = 0; c < S::U; ++c) w[c] = a[c];
+    }
+    if (alpha_mode == 1) {
+      alpha_t[t] = alpha_in[t];
+    } else if (alpha_mode >= 2) {
+      // convexity shift bound beta(A) <= (m-1) sum_{i_1..i_m} |a| = (m-1) sum_c (m!/k!) |a_c| (R17)
+      float b = 0.f;
+      static_for<S::U>([&](auto cc) {
+        constexpr int c = decltype(cc)::value;
+        constexpr float mult = (float)S::T.cls_mult[c];
+        b = fmaf(mult, fabsf(a[c]), b);
+      });
+      b *= (float)(M - 1);
+      alpha_t[t] = (alpha_mode == 2) ? b : -b;
     }
     float4* dst = packed + t * (S::PW / 4);
 #pragma unroll
@@ -281,6 +295,7 @@ struct SolveParams {
   int S;
   FastDiv divS;
   float alpha, tol;
+  const float* alpha_t;      // SHIFT == 3: per-tensor shift [N] (from the pack kernel)
   int maxit;
   int refill_k;              // refill threshold
   // fused solve -> dedup (FUSED kernels only)
@@ -301,7 +316,8 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return r;
 }
 
-// SHIFT: 0 -> alpha == 0 (xhat = g), 1 -> alpha > 0 (xhat = g + alpha x), 2 -> alpha < 0 (xhat = -(g + alpha x))
+// SHIFT: 0 -> alpha == 0 (xhat = g), 1 -> alpha > 0 (xhat = g + alpha x), 2 -> alpha < 0 (xhat = -(g + alpha x)),
+//        3 -> per-tensor alpha from p.alpha_t (schedule 1 only)
 // WIDE: 64-bit item indices (N*S >= 2^31); otherwise 32-bit index arithmetic.
 // FUSED: also cluster each chunk's tensors (R16) as soon as the warp has
 // written the chunk's last item (open chunks tracked in a shared-memory ring;
@@ -354,6 +370,7 @@ sshopm_solve_kernel(const SolveParams p) {
   int k = 0;
   bool has = false, stop = true, conv = false;
   Idx item = 0;
+  float la = 0.f, ls = 1.f;  // SHIFT == 3: per-lane |alpha| and sign: xhat = ls*g + la*x
   unsigned long long it_sum = 0;
 
   for (;;) {
@@ -415,6 +432,11 @@ sshopm_solve_kernel(const SolveParams p) {
         const uint32_t s = t - vq * S_;
         item = v0 * (Idx)S_ + (Idx)t;
         if constexpr (FUSED) cseq = cur ? cur_seq : claim_seq;
+        if constexpr (SHIFT == 3) {
+          const float at = __ldg(p.alpha_t + (v0 + (Idx)vq));
+          ls = at >= 0.f ? 1.f : -1.f;                     // Fig. 1 lines 2-5 (R5: alpha = 0 -> "+")
+          la = fabsf(at);
+        }
         cf.load(p.packed + (v0 + (Idx)vq) * (Idx)(S::PW / 4));
         float v[4 * SST4];
 #pragma unroll
@@ -487,13 +509,15 @@ sshopm_solve_kernel(const SolveParams p) {
         constexpr int i = decltype(qq)::value;
         if constexpr (SHIFT == 0) hp[i] = gp[i];
         else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
-        else hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
+        else if constexpr (SHIFT == 2) hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
+        else hp[i] = __ffma2_rn(bc(la), xs[i], __fmul2_rn(gp[i], bc(ls)));
       });
       if constexpr (S::ODD) {
         float h;
         if constexpr (SHIFT == 0) h = gs;
         else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
-        else h = fmaf(alpha, xs[S::NX - 1].x, -gs);
+        else if constexpr (SHIFT == 2) h = fmaf(alpha, xs[S::NX - 1].x, -gs);
+        else h = fmaf(la, xs[S::NX - 1].x, gs * ls);
         hp[S::NX - 1] = f2(h, 0.f);
       }
       float nn;

@@ -70,14 +70,21 @@ struct Tables {
   int q_right[Q];                 // lower-list index of the degree-H suffix (-1 if H == 0)
   int q_cls[Q][N];                // class position of q + e_j
   long long q_coef[Q];            // (M-1)! / q!
+  long long cls_mult[U];          // M! / k! : tensor indices in class c (Property 2)
   int n_products;                 // FP32 multiplies to form the Q monomials (no coefficient)
 
-  constexpr Tables() : cls_idx(), deg_off(), low_parent(), low_var(), q_left(), q_right(), q_cls(), q_coef(), n_products(0) {
+  constexpr Tables() : cls_idx(), deg_off(), low_parent(), low_var(), q_left(), q_right(), q_cls(), q_coef(), cls_mult(), n_products(0) {
     // classes of degree M in lex order
     {
       int I[M > 0 ? M : 1] = {};
       for (int c = 0; c < U; ++c) {
-        for (int t = 0; t < M; ++t) cls_idx[c][t] = I[t];
+        long long den = 1;
+        int run = 1;
+        for (int t = 0; t < M; ++t) {
+          cls_idx[c][t] = I[t];
+          if (t > 0 && I[t] == I[t - 1]) { ++run; den *= run; } else run = 1;
+        }
+        cls_mult[c] = fact(M) / den;
         next_tuple(I, M, N);
       }
     }

@@ -53,8 +53,13 @@ def angle(a, b, even):
     return t
 
 
+def _lane_alpha(alpha, vox):
+    """Scalar shift, or the per-voxel shift array indexed for these lanes."""
+    return alpha if np.ndim(alpha) == 0 else np.asarray(alpha, np.float64)[vox]
+
+
 def _lanes(full, vox, x0, alpha, tol, maxit, lane_maxit=None, dtype=np.float64):
-    return O.sshopm_lanes(lambda idx: full[vox[idx]], x0, alpha, tol, maxit, lane_maxit, dtype=dtype)
+    return O.sshopm_lanes(lambda idx: full[vox[idx]], x0, _lane_alpha(alpha, vox), tol, maxit, lane_maxit, dtype=dtype)
 
 
 def _perturb(x0, seed, k):
@@ -78,7 +83,7 @@ def _history(full, vox, x0, alpha, K, dtype=np.float64):
     h[0] = O.axm(full[vox], x0.astype(dtype), dtype)
     hx[0] = x0
     tr = []
-    O.sshopm_lanes(lambda idx: full[vox[idx]], x0, alpha, -1.0, K, trace=tr, dtype=dtype)
+    O.sshopm_lanes(lambda idx: full[vox[idx]], x0, _lane_alpha(alpha, vox), -1.0, K, trace=tr, dtype=dtype)
     for kk, ids, ln, xn in tr:
         h[kk, ids] = ln
         hx[kk, ids] = xn

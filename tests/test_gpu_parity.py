@@ -302,3 +302,46 @@ def test_fused_ring_overflow(dev):
     assert ra[2].max() == 3000 and (ra[2] == 3000).sum() > 100    # slow lanes really ran to maxit
     for a, b in zip(ra + da, rb + db):
         assert np.array_equal(a, b)
+
+
+# --------------------------------------------------------------- shift modes --
+def test_per_tensor_alpha_parity(dev):
+    """alpha_mode 1: one shift per tensor (mixed signs) vs the oracle with the same per-voxel shifts."""
+    m, n, V = 4, 3, 256
+    ent = syn.gen_voxels(m, n, 4242, V, 0)
+    st = syn.gen_starts(128, n, 0)
+    rng = np.random.default_rng(3)
+    al = rng.choice([0.0, 0.25, 0.5, 1.0, -0.5], size=V).astype(np.float32)
+    s = sh.Solver(m, n)
+    out = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), torch.from_numpy(al).to(dev), 1e-6, 100)
+    torch.cuda.synchronize()
+    gpu = tuple(t.cpu().numpy() for t in out)
+    _assert_parity(PR.solve_parity(ent, st, m, n, al.astype(np.float64), 1e-6, 100, gpu), 0.02)
+    # a constant array equals the scalar path bit for bit
+    c = torch.full((V,), 0.5, dtype=torch.float32, device=dev)
+    a1 = [t.cpu().numpy() for t in s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), c, 1e-6, 100)]
+    a2 = [t.cpu().numpy() for t in s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.5, 1e-6, 100)]
+    for a, b in zip(a1, a2):
+        assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("mode,sign", [("auto_max", 1.0), ("auto_min", -1.0)])
+def test_auto_shift_monotone_and_parity(dev, mode, sign):
+    """alpha = +-(m-1) sum|a| (R17): every GPU lambda trajectory is monotone, all lanes converge,
+    and results match the oracle run with its own independently computed shift."""
+    from oracle import sshopm as OR
+    m, n, V = 4, 3, 64
+    ent = syn.gen_uniform_tensors(m, n, V, 8)            # unstructured: alpha = 0 would often fail
+    st = syn.gen_starts(32, n, 2)
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    prev = None
+    for K in range(0, 30):
+        lamK = s.solve(e, t, mode, -1.0, K)[0].cpu().numpy()
+        if prev is not None:
+            assert np.all(sign * (lamK - prev) >= -2e-5 * np.maximum(1, np.abs(prev)))
+        prev = lamK
+    lam, x, it, cv = (u.cpu().numpy() for u in s.solve(e, t, mode, 1e-6, 2000))
+    assert cv.mean() > 0.99
+    al = sign * OR.convexity_shift(ent, m, n)
+    _assert_parity(PR.solve_parity(ent, st, m, n, al, 1e-6, 2000, (lam, x, it, cv)), 0.02)

@@ -251,3 +251,37 @@ def test_paper_flops_reading_r12():
     """R12 (parity unpinned): F(4,3) = 6*15 + 5*30 + 15 = 255."""
     assert O.paper_flops_per_iter(4, 3) == 255
     assert O.paper_flops_per_iter(6, 3) == 680
+
+
+def test_per_voxel_alpha_equals_scalar_runs():
+    """A per-voxel shift array gives exactly the per-voxel scalar runs (incl. mixed signs)."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 6, seed=2)
+    st = syn.gen_starts(32, n, 1)
+    alphas = np.array([0.0, 0.5, -0.5, 2.0, -2.0, 0.25])
+    lam, x, it, cv = _run(ent, st, m, n, alphas, 1e-8, 200)
+    for v in range(6):
+        l1, x1, i1, c1 = _run(ent[v:v + 1], st, m, n, float(alphas[v]), 1e-8, 200)
+        assert np.array_equal(lam[v], l1[0]) and np.array_equal(x[v], x1[0]) and np.array_equal(it[v], i1[0])
+
+
+def test_convexity_shift_bound_and_monotone():
+    """R17 shift: brute-force sum over all n^m entries; lambda_k nondecreasing (+) / nonincreasing (-)."""
+    m, n = 4, 3
+    ent = syn.gen_uniform_tensors(m, n, 4, seed=5).astype(np.float64)
+    b = O.convexity_shift(ent, m, n)
+    full = O.expand_full(ent, m, n)
+    for v in range(4):
+        import itertools
+        tot = sum(abs(full[v][t]) for t in itertools.product(range(n), repeat=m))
+        assert np.isclose(b[v], (m - 1) * tot)
+    for sign in (1, -1):
+        x0 = O.normalise_starts(syn.gen_starts(16, n, 3))
+        fl = full[0:1]
+        lam0 = O.axm(np.repeat(fl, 16, 0), x0)
+        tr = []
+        O.sshopm_lanes(lambda idx: fl[np.zeros(len(idx), int)], x0, sign * b[0], -1.0, 25, trace=tr)
+        prev = lam0.copy()
+        for k, ids, ln, _ in tr:
+            assert np.all(sign * (ln - prev[ids]) >= -1e-12)
+            prev[ids] = ln
