@@ -5,10 +5,12 @@
 #include <stdint.h>
 #include "launchers.h"
 
-namespace sshopm { struct HostCache; }
+namespace sshopm { struct HostCache; struct GeneralTables; }
 
 struct sshopm_ctx {
-  const sshopm::Launchers* L;
+  const sshopm::Launchers* L;      // compiled (m, n) kernels, or null
+  sshopm::GeneralTables* gen;      // table-driven kernel tables (any (m, n))
+  int m, n, U;
   std::atomic<long long> launches;
   sshopm::HostCache* hc;     // run_host device buffers / streams (created lazily, guarded by its mutex)
 };
@@ -29,16 +31,17 @@ struct Workspace {
   bool owned = false;
 };
 size_t workspace_bytes(const Launchers* L, int64_t N, int S);
+size_t handle_workspace_bytes(const sshopm_ctx* h, int64_t N, int S);
 int acquire_workspace(const Launchers* L, int64_t N, int S, void* user, size_t user_bytes, cudaStream_t st, Workspace* ws);
 int release_workspace(Workspace* ws, cudaStream_t st);
-int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
+int dedup_impl(int m, int n, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
                float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
                int32_t* d_rep, cudaStream_t st);
 void free_host_cache(sshopm_ctx* h);
 int chunk_tensors_for(int S);
-int make_dedup_params(const Launchers* L, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
+int make_dedup_params(int n, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
                       float* d_olam, float* d_ox, int32_t* d_mult, int32_t* d_rep, DedupParams* p);
-int launch_dedup(const Launchers* L, const DedupParams& p, cudaStream_t st);
-int launch_dedup_list(const Launchers* L, const DedupParams& p, const unsigned int* count, const unsigned int* list,
+int launch_dedup(int m, int n, const DedupParams& p, cudaStream_t st);
+int launch_dedup_list(int m, int n, const DedupParams& p, const unsigned int* count, const unsigned int* list,
                       int chunk_tensors, cudaStream_t st);
 }  // namespace sshopm

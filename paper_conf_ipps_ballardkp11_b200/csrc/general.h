@@ -1,0 +1,28 @@
+// general.h — table-driven kernel for any (m, n) (general.cu).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include "sshopm.h"
+
+namespace sshopm {
+
+constexpr int kGenMaxM = 16;     // order limit of the general kernel
+constexpr int kGenMaxN = 16;     // dimension limit
+constexpr long long kGenMaxU = 1 << 16;
+
+struct GeneralTables {           // host copies; uploaded per call (handles own no device memory)
+  int m = 0, n = 0, U = 0;
+  uint8_t* idx = nullptr;        // [U][m] index representations, lexicographic (Fig. 4 walk)
+  int* mult = nullptr;           // [U] m!/k! (Property 2)
+  long long paper_flops = 0, exec_flops = 0;
+};
+
+GeneralTables* general_create(int m, int n);
+void general_destroy(GeneralTables* t);
+int general_solve(const GeneralTables* t, int64_t N, const float* d_entries, int S, const float* d_starts, float alpha,
+                  float tol, int maxit, float* d_lambda, float* d_x, int32_t* d_iters, uint8_t* d_conv,
+                  const sshopm_solve_opts* opts, cudaStream_t st);
+int general_apply(const GeneralTables* t, int64_t N, const float* d_entries, const float* d_x, float* d_g, float* d_lam,
+                  cudaStream_t st);
+
+}  // namespace sshopm

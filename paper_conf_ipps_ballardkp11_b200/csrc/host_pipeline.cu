@@ -78,7 +78,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   if (!h_entries || !h_starts || !h_out_count || !h_out_lambda || !h_out_x || !h_out_mult) return SSHOPM_EINVAL;
   const bool raw = h_raw_lambda || h_raw_x || h_raw_iters || h_raw_converged;
   if (raw && !(h_raw_lambda && h_raw_x && h_raw_iters && h_raw_converged)) return SSHOPM_EINVAL;
-  const int n = h->L->n, U = h->L->U;
+  const int n = h->n, U = h->U;
   long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 32;   // default: ~32 chunks, 4K..64K tensors
   if (chunk_tensors <= 0) chunk = chunk < 4096 ? 4096 : (chunk > 65536 ? 65536 : chunk);
   if (chunk > N) chunk = N;
@@ -119,7 +119,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
       CK(cudaMalloc(&s.ox, sizeof(float) * chunk * kmax * n), "run_host: malloc");
       CK(cudaMalloc(&s.mult, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
       CK(cudaMalloc(&s.rep, sizeof(int32_t) * chunk * kmax), "run_host: malloc");
-      s.ws_bytes = workspace_bytes(h->L, chunk, S);
+      s.ws_bytes = handle_workspace_bytes(h, chunk, S);
       CK(cudaMalloc(&s.ws, s.ws_bytes), "run_host: malloc");
     }
     c->chunk = chunk;

@@ -14,6 +14,7 @@
 #include "sshopm.h"
 #include "sshopm_dedup.cuh"
 #include "api_internal.h"
+#include "general.h"
 
 namespace sshopm {
 #define SHAPE(mm, nn) const Launchers* get_launchers_##mm##_##nn();
@@ -47,6 +48,10 @@ FastDiv make_fastdiv(uint32_t d) {
 static size_t starts_region(const Launchers* L, int S) {
   const size_t b = (size_t)S * (size_t)((L->n + 3) / 4 * 4) * 4;
   return (b + 255) / 256 * 256;
+}
+
+size_t handle_workspace_bytes(const sshopm_ctx* h, int64_t N, int S) {
+  return h->L ? workspace_bytes(h->L, N, S) : 256;          // the general kernel needs no workspace
 }
 
 int chunk_tensors_for(int S) { return (S >= 256) ? 1 : (256 + S - 1) / S; }
@@ -125,7 +130,7 @@ const char* sshopm_supported_shapes(void) {
 #define SHAPE(mm, nn) #mm "x" #nn ","
 #include "shapes.def"
 #undef SHAPE
-      "";
+      "";   // compiled (unrolled) shapes; any other m <= 16, n <= 16 uses the table-driven general kernel
   return s;
 }
 
@@ -133,10 +138,15 @@ int sshopm_create(int m, int n, sshopm_t* out) {
   if (!out || m < 2 || n < 1) return SSHOPM_EINVAL;
   *out = nullptr;
   const Launchers* L = find_launchers(m, n);
-  if (!L) return SSHOPM_EUNSUPPORTED;
+  GeneralTables* gen = general_create(m, n);                 // also backs opts.schedule = 3 on compiled shapes
+  if (!L && !gen) return SSHOPM_EUNSUPPORTED;
   sshopm_ctx* h = new (std::nothrow) sshopm_ctx;
-  if (!h) return SSHOPM_ENOMEM;
+  if (!h) { general_destroy(gen); return SSHOPM_ENOMEM; }
   h->L = L;
+  h->gen = gen;
+  h->m = m;
+  h->n = n;
+  h->U = L ? L->U : gen->U;
   h->launches.store(0);
   h->hc = nullptr;
   *out = h;
@@ -145,26 +155,28 @@ int sshopm_create(int m, int n, sshopm_t* out) {
 
 int sshopm_destroy(sshopm_t h) {
   if (h) free_host_cache(h);
+  if (h) general_destroy(h->gen);
   delete h;
   return SSHOPM_OK;
 }
 
 int sshopm_num_unique(sshopm_t h, int* U) {
   if (!h || !U) return SSHOPM_EINVAL;
-  *U = h->L->U;
+  *U = h->U;
   return SSHOPM_OK;
 }
 
 int sshopm_class_index(sshopm_t h, int32_t* h_idx) {
   if (!h || !h_idx) return SSHOPM_EINVAL;
-  h->L->class_index(h_idx);
+  if (h->L) h->L->class_index(h_idx);
+  else for (int i = 0; i < h->U * h->m; ++i) h_idx[i] = h->gen->idx[i];
   return SSHOPM_OK;
 }
 
 int sshopm_flops_per_iter(sshopm_t h, int64_t* paper, int64_t* executed) {
   if (!h) return SSHOPM_EINVAL;
-  if (paper) *paper = h->L->paper_flops;
-  if (executed) *executed = h->L->exec_flops;
+  if (paper) *paper = h->L ? h->L->paper_flops : h->gen->paper_flops;
+  if (executed) *executed = h->L ? h->L->exec_flops : h->gen->exec_flops;
   return SSHOPM_OK;
 }
 
@@ -176,7 +188,7 @@ int sshopm_launch_count(sshopm_t h, int64_t* count) {
 
 int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes) {
   if (!h || N < 0 || S < 0 || !bytes) return SSHOPM_EINVAL;
-  *bytes = workspace_bytes(h->L, N, S);
+  *bytes = handle_workspace_bytes(h, N, S);
   return SSHOPM_OK;
 }
 
@@ -196,6 +208,22 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const Launchers* L = h->L;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
+  if (!L || (opts && opts->schedule == 3)) {                     // table-driven general kernel (any (m, n))
+    if (!h->gen) return SSHOPM_EUNSUPPORTED;
+    int rc = general_solve(h->gen, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
+                           d_out_converged, opts, st);
+    if (rc != SSHOPM_OK) return rc;
+    h->launches.fetch_add(1);
+    if (dd) {
+      DedupParams q = *dd;
+      q.lambda = d_out_lambda;
+      q.x = d_out_x;
+      q.conv = d_out_converged;
+      rc = launch_dedup(h->m, h->n, q, st);
+      if (rc == SSHOPM_OK) h->launches.fetch_add(1);
+    }
+    return rc;
+  }
 
   // shift: scalar alpha (R4), or per tensor (alpha_mode 1: caller's array; 2 / 3: +- convexity bound, R17)
   const int alpha_mode = opts ? opts->alpha_mode : 0;
@@ -205,7 +233,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const bool wide = (long long)N * S >= (1LL << 31) - (1LL << 20);
   // schedule: 1 = item per lane (chunks of whole tensors), 2 = tensor per lane
   int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
-  if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;
+  if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;   // 3 (general) handled above
   if (shift == 3) schedule = 1;                                  // per-tensor alpha: schedule 1 only
   int bps = 0;
   cudaError_t e = L->occupancy(shift, wide, schedule, 0, 0, &bps);
@@ -278,8 +306,8 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
   h->launches.fetch_add(2);
   if (dd) {
-    if (fused) rc = launch_dedup_list(L, p.dd, ws.ovf_count, ws.ovf_list, chunk_tensors, st);
-    else rc = launch_dedup(L, p.dd, st);
+    if (fused) rc = launch_dedup_list(h->m, h->n, p.dd, ws.ovf_count, ws.ovf_list, chunk_tensors, st);
+    else rc = launch_dedup(h->m, h->n, p.dd, st);
     if (rc != SSHOPM_OK) { release_workspace(&ws, st); return rc; }
     h->launches.fetch_add(1);
   }
@@ -305,7 +333,7 @@ int sshopm_solve_dedup(sshopm_t h, int64_t N, const float* d_entries, int S, con
                        int32_t* d_out_rep, const sshopm_solve_opts* opts, void* stream) {
   if (!h) return SSHOPM_EINVAL;
   DedupParams dd;
-  int rc = make_dedup_params(h->L, N, S, lam_tol, ang_tol, kmax, d_out_count, d_out_clambda, d_out_cx, d_out_mult,
+  int rc = make_dedup_params(h->n, N, S, lam_tol, ang_tol, kmax, d_out_count, d_out_clambda, d_out_cx, d_out_mult,
                              d_out_rep, &dd);
   if (rc != SSHOPM_OK) return rc;
   return solve_impl(h, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
@@ -328,6 +356,11 @@ int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x
   cudaStream_t st = (cudaStream_t)stream;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_apply: no device");
+  if (!h->L) {
+    int rc = general_apply(h->gen, N, d_entries, d_x, d_out_g, d_out_lam, st);
+    if (rc == SSHOPM_OK) h->launches.fetch_add(1);
+    return rc;
+  }
   long long grid = (N + 255) / 256;
   if (grid > (long long)sms * 16) grid = (long long)sms * 16;
   Workspace ws;
@@ -363,12 +396,12 @@ static cudaError_t launch_dedup128(const DedupParams& p, int grid, int block, in
   return cudaGetLastError();
 }
 
-int make_dedup_params(const Launchers* L, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
+int make_dedup_params(int n, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
                       float* d_olam, float* d_ox, int32_t* d_mult, int32_t* d_rep, DedupParams* p) {
   if (S < 1 || kmax < 1 || !(lam_tol >= 0.f) || !(ang_tol >= 0.f) || N < 0) return SSHOPM_EINVAL;
   if (N > 0 && (!d_count || !d_olam || !d_ox || !d_mult)) return SSHOPM_EINVAL;
   if (S > 1024) return SSHOPM_EUNSUPPORTED;
-  if (L->n > 8) return SSHOPM_EUNSUPPORTED;
+  if (n > 8) return SSHOPM_EUNSUPPORTED;
   p->lambda = nullptr;
   p->x = nullptr;
   p->conv = nullptr;
@@ -385,10 +418,10 @@ int make_dedup_params(const Launchers* L, int64_t N, int S, float lam_tol, float
   return SSHOPM_OK;
 }
 
-static int dedup_launch_shape(const Launchers* L, int64_t N, int S, bool fast, int* grid, int* block, int* smem) {
+static int dedup_launch_shape(int n, int64_t N, int S, bool fast, int* grid, int* block, int* smem) {
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_dedup: no device");
-  const int per_warp = fast ? 128 * (L->n + 3) * 4 : dedup_smem_words(S, L->n) * 4;
+  const int per_warp = fast ? 128 * (n + 3) * 4 : dedup_smem_words(S, n) * 4;
   int wpb = (96 * 1024) / per_warp;
   if (wpb > 8) wpb = 8;
   if (wpb < 1) wpb = 1;
@@ -401,16 +434,16 @@ static int dedup_launch_shape(const Launchers* L, int64_t N, int S, bool fast, i
   return SSHOPM_OK;
 }
 
-int launch_dedup(const Launchers* L, const DedupParams& p, cudaStream_t st) {
+int launch_dedup(int m, int n, const DedupParams& p, cudaStream_t st) {
   if (p.n_tensors == 0) return SSHOPM_OK;
   if (!p.lambda || !p.x || !p.conv) return SSHOPM_EINVAL;
-  const int S = p.S, n = L->n;
+  const int S = p.S;
   const bool fast = (S == 128) && ((uintptr_t)p.lambda % 16 == 0) && ((uintptr_t)p.x % 16 == 0) &&
                     ((uintptr_t)p.conv % 4 == 0);
   int grid, block, smem;
-  int rc = dedup_launch_shape(L, p.n_tensors, S, fast, &grid, &block, &smem);
+  int rc = dedup_launch_shape(n, p.n_tensors, S, fast, &grid, &block, &smem);
   if (rc != SSHOPM_OK) return rc;
-  const bool even = (L->m % 2) == 0;
+  const bool even = (m % 2) == 0;
   cudaError_t e = cudaErrorInvalidValue;
   switch (n) {
 #define DD(NN) case NN: e = fast ? (even ? launch_dedup128<NN, true>(p, grid, block, smem, st) : launch_dedup128<NN, false>(p, grid, block, smem, st)) \
@@ -434,16 +467,16 @@ static cudaError_t launch_list_t(const DedupParams& p, const unsigned int* count
   return cudaGetLastError();
 }
 
-int launch_dedup_list(const Launchers* L, const DedupParams& p, const unsigned int* count, const unsigned int* list,
+int launch_dedup_list(int m, int n, const DedupParams& p, const unsigned int* count, const unsigned int* list,
                       int chunk_tensors, cudaStream_t st) {
   int grid, block, smem;
-  int rc = dedup_launch_shape(L, p.n_tensors, p.S, false, &grid, &block, &smem);
+  int rc = dedup_launch_shape(n, p.n_tensors, p.S, false, &grid, &block, &smem);
   if (rc != SSHOPM_OK) return rc;
   const int sms = device_sms();
   if (grid > sms * 2) grid = sms * 2;                     // untracked chunks are rare
-  const bool even = (L->m % 2) == 0;
+  const bool even = (m % 2) == 0;
   cudaError_t e = cudaErrorInvalidValue;
-  switch (L->n) {
+  switch (n) {
 #define DD(NN) case NN: e = even ? launch_list_t<NN, true>(p, count, list, chunk_tensors, grid, block, smem, st) \
                              : launch_list_t<NN, false>(p, count, list, chunk_tensors, grid, block, smem, st); break;
     DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
@@ -454,18 +487,18 @@ int launch_dedup_list(const Launchers* L, const DedupParams& p, const unsigned i
   return SSHOPM_OK;
 }
 
-int dedup_impl(const Launchers* L, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
+int dedup_impl(int m, int n, int64_t N, int S, const float* d_lambda, const float* d_x, const uint8_t* d_conv,
                float lam_tol, float ang_tol, int kmax, int32_t* d_count, float* d_olam, float* d_ox, int32_t* d_mult,
                int32_t* d_rep, cudaStream_t st) {
   DedupParams p;
-  int rc = make_dedup_params(L, N, S, lam_tol, ang_tol, kmax, d_count, d_olam, d_ox, d_mult, d_rep, &p);
+  int rc = make_dedup_params(n, N, S, lam_tol, ang_tol, kmax, d_count, d_olam, d_ox, d_mult, d_rep, &p);
   if (rc != SSHOPM_OK) return rc;
   if (N == 0) return SSHOPM_OK;
   if (!d_lambda || !d_x || !d_conv) return SSHOPM_EINVAL;
   p.lambda = d_lambda;
   p.x = d_x;
   p.conv = d_conv;
-  return launch_dedup(L, p, st);
+  return launch_dedup(m, n, p, st);
 }
 }  // namespace sshopm
 
@@ -475,7 +508,7 @@ extern "C" int sshopm_dedup(sshopm_t h, int64_t N, int S,
                             int32_t* d_out_count, float* d_out_lambda, float* d_out_x, int32_t* d_out_mult,
                             int32_t* d_out_rep, void* stream) {
   if (!h) return SSHOPM_EINVAL;
-  int r = dedup_impl(h->L, N, S, d_lambda, d_x, d_converged, lam_tol, ang_tol, kmax, d_out_count, d_out_lambda,
+  int r = dedup_impl(h->m, h->n, N, S, d_lambda, d_x, d_converged, lam_tol, ang_tol, kmax, d_out_count, d_out_lambda,
                      d_out_x, d_out_mult, d_out_rep, (cudaStream_t)stream);
   if (r == SSHOPM_OK && N > 0) h->launches.fetch_add(1);
   return r;

@@ -345,3 +345,45 @@ def test_auto_shift_monotone_and_parity(dev, mode, sign):
     assert cv.mean() > 0.99
     al = sign * OR.convexity_shift(ent, m, n)
     _assert_parity(PR.solve_parity(ent, st, m, n, al, 1e-6, 2000, (lam, x, it, cv)), 0.02)
+
+
+# ------------------------------------------------------- general (table) kernel --
+@pytest.mark.parametrize("m,n", [(5, 4), (7, 2), (3, 6), (9, 3), (4, 3)])
+def test_general_apply_exact(dev, m, n):
+    """Table-driven Eq. 6 (any (m, n)) is bit-exact on small integers like the unrolled kernels."""
+    ent, x = _exact_inputs(m, n, 300, m * 11 + n)
+    if m >= 7:
+        ent = np.clip(ent, -2, 2)
+    full = O.expand_full(ent, m, n)
+    g_ref = O.axm1(full, x.astype(np.float64))
+    lam_ref = O.axm(full, x.astype(np.float64))
+    assert np.abs(g_ref).max() < 2 ** 24 and np.abs(lam_ref).max() < 2 ** 24
+    s = sh.Solver(m, n)
+    if (m, n) in set(sh.supported_shapes()):
+        pytest.skip("compiled shape: apply uses the unrolled kernel")
+    g, lam = s.apply(torch.from_numpy(ent).to(dev), torch.from_numpy(x).to(dev))
+    assert np.array_equal(g.cpu().numpy().astype(np.float64), g_ref)
+    assert np.array_equal(lam.cpu().numpy().astype(np.float64), lam_ref)
+
+
+@pytest.mark.parametrize("m,n,V,alpha", [(5, 4, 24, 4.0), (6, 4, 16, 0.5), (3, 6, 16, 3.0), (10, 2, 32, 0.5), (4, 8, 8, 0.0)])
+def test_general_solve_parity(dev, m, n, V, alpha):
+    ent = syn.gen_voxels(m, n, 0, V, 3) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 3)
+    st = syn.gen_starts(64, n, 1)
+    gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 200)
+    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 200, gpu), 0.05)
+
+
+def test_general_kernel_on_compiled_shape(dev):
+    """opts.schedule = 3 forces the table-driven kernel on (4,3): same contract vs the oracle."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 256, 0)
+    st = syn.gen_starts(128, n, 0)
+    gpu = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, schedule=3)
+    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, gpu))
+    # automatic shift: the general and unrolled kernels agree (different FP32 summation orders)
+    a3 = _solve(dev, m, n, ent[:32], st, "auto_max", 1e-6, 300, schedule=3)
+    a1 = _solve(dev, m, n, ent[:32], st, "auto_max", 1e-6, 300, schedule=1)
+    both = (a3[3] == 1) & (a1[3] == 1)
+    assert both.mean() > 0.5
+    assert np.all(np.abs(a3[0][both] - a1[0][both]) <= 1e-4 * np.maximum(1, np.abs(a1[0][both])))

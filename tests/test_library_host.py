@@ -40,10 +40,11 @@ def test_create_errors():
     assert L.sshopm_create(1, 3, ctypes.byref(h)) == sh.EINVAL
     assert L.sshopm_create(4, 0, ctypes.byref(h)) == sh.EINVAL
     assert L.sshopm_create(4, 3, None) == sh.EINVAL
-    assert L.sshopm_create(9, 9, ctypes.byref(h)) == sh.EUNSUPPORTED
+    assert L.sshopm_create(17, 3, ctypes.byref(h)) == sh.EUNSUPPORTED      # beyond the general kernel's m <= 16
+    assert L.sshopm_create(4, 17, ctypes.byref(h)) == sh.EUNSUPPORTED
     assert L.sshopm_destroy(None) == sh.OK
     with pytest.raises(sh.SSHOPMError):
-        sh.Solver(7, 7)
+        sh.Solver(20, 20)
 
 
 def test_status_strings():
@@ -91,4 +92,15 @@ def test_host_side_argument_validation():
     assert L.sshopm_dedup(s._h, 10, 2048, dummy, dummy, dummy, 0.01, 0.05, 4, *d5, None) == sh.EUNSUPPORTED
     assert L.sshopm_apply(s._h, 0, None, None, None, None, None) == sh.OK
     assert L.sshopm_apply(s._h, 3, None, None, None, None, None) == sh.EINVAL
+    s.close()
+
+
+@pytest.mark.parametrize("m,n", [(5, 4), (7, 2), (3, 6), (9, 3), (2, 9), (6, 5), (10, 2)])
+def test_general_shapes_tables(m, n):
+    """(m, n) without a compiled kernel: the general kernel's Fig. 4 tables equal the oracle's enumeration."""
+    assert (m, n) not in set(sh.supported_shapes())
+    s = sh.Solver(m, n)
+    assert s.U == O.num_unique(m, n)
+    assert np.array_equal(s.class_index(), np.array(O.class_list(m, n), dtype=np.int32))
+    assert s.paper_flops_per_iter == O.paper_flops_per_iter(m, n)
     s.close()
