@@ -168,6 +168,17 @@ int sshopm_solve_dedup(sshopm_t h, int64_t N, const float* d_entries, int S, con
                        int32_t* d_out_count, float* d_out_clambda, float* d_out_cx, int32_t* d_out_mult,
                        int32_t* d_out_rep, const sshopm_solve_opts* opts, void* stream);
 
+/* Eigenpair type of each dedup record (reading R18; fibre directions are the
+ * local maxima of A g^m on the sphere).  For record
+ * k of tensor t (k < count[t]) with (lam, x) = (d_lambda[t][k], d_x[t][k]):
+ * C = U^T [(m-1) A x^{m-2} - lam I] U on x-perp (Definition 2 with p = 2);
+ * d_out_type[t][k] = +1 local maximum (C negative definite), -1 local minimum,
+ * 0 saddle, 2 degenerate (an eigenvalue of C within ctol * max(1, |lam|) of 0),
+ * 3 empty slot (k >= count[t]).  Inputs are sshopm_dedup's outputs and the
+ * tensors' entries.  Compiled (m, n) only (else EUNSUPPORTED). */
+int sshopm_classify(sshopm_t h, int64_t N, const float* d_entries, int kmax, const int32_t* d_count,
+                    const float* d_lambda, const float* d_x, float ctol, int8_t* d_out_type, void* stream);
+
 /* Test hook: d_out_g[N][n] = A x^{m-1} (Eq. 6) and d_out_lam[N] = A x^m
  * (Eq. 4 via Euler's identity x.(A x^{m-1})) for N (tensor, x) pairs, using
  * exactly the solver's compiled evaluation.  d_x[N][n] is NOT normalised. */

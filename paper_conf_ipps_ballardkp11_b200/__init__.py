@@ -62,6 +62,7 @@ def lib():
         "sshopm_solve_dedup": (I, [P, I64, P, I, P, F, F, I, P, P, P, P, F, F, I, P, P, P, P, P,
                                    ctypes.POINTER(_Opts), P]),
         "sshopm_apply": (I, [P, I64, P, P, P, P, P]),
+        "sshopm_classify": (I, [P, I64, P, I, P, P, P, F, P, P]),
         "sshopm_run_host": (I, [P, I64, P, I, P, F, F, I, F, F, I, P, P, P, P, P, P, P, P, P, I64, P]),
         "sshopm_launch_count": (I, [P, ctypes.POINTER(I64)]),
         "sshopm_workspace_size": (I, [P, I64, I, ctypes.POINTER(ctypes.c_size_t)]),
@@ -270,6 +271,17 @@ class Solver:
                                   _dev(ox, torch.float32, (N, kmax, self.n), "out_x"),
                                   _dev(om, torch.int32, (N, kmax), "out_mult"),
                                   _dev(orp, torch.int32, (N, kmax), "out_rep"), _stream(stream)), "sshopm_dedup")
+        return out
+
+    def classify(self, entries, count, lam, x, ctol=1e-3, stream=None):
+        """Eigenpair types [N, kmax] int8 of dedup records: +1 max, -1 min, 0 saddle, 2 degenerate, 3 empty."""
+        torch = _torch()
+        N, K = int(lam.shape[0]), int(lam.shape[1])
+        out = torch.empty((N, K), dtype=torch.int8, device=lam.device)
+        _check(lib().sshopm_classify(self._h, N, _dev(entries, torch.float32, (N, self.U), "entries"), K,
+                                     _dev(count, torch.int32, (N,), "count"), _dev(lam, torch.float32, (N, K), "lambda"),
+                                     _dev(x, torch.float32, (N, K, self.n), "x"), float(ctol),
+                                     ctypes.c_void_p(out.data_ptr()), _stream(stream)), "sshopm_classify")
         return out
 
     def apply(self, entries, x, stream=None):

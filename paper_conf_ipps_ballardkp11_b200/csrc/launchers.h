@@ -19,6 +19,8 @@ struct Launchers {
                       int grid, cudaStream_t st);
   cudaError_t (*solve)(const SolveParams& p, int shift, bool wide, int schedule, int fused, int grid, int smem_bytes,
                        cudaStream_t st);
+  cudaError_t (*classify)(long long n_tensors, int kmax, const float* entries, const int32_t* count, const float* lam,
+                          const float* x, float ctol, int8_t* out, int grid, cudaStream_t st);
   cudaError_t (*apply)(long long n_items, const float4* packed, const float* x, float* g, float* lam, int grid,
                        cudaStream_t st);
 };

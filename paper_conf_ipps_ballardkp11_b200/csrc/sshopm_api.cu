@@ -348,6 +348,23 @@ int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const flo
                          d_out_converged, nullptr, stream);
 }
 
+int sshopm_classify(sshopm_t h, int64_t N, const float* d_entries, int kmax, const int32_t* d_count,
+                    const float* d_lambda, const float* d_x, float ctol, int8_t* d_out_type, void* stream) {
+  if (!h || N < 0 || kmax < 1 || !(ctol >= 0.f)) return SSHOPM_EINVAL;
+  if (N == 0) return SSHOPM_OK;
+  if (!d_entries || !d_count || !d_lambda || !d_x || !d_out_type) return SSHOPM_EINVAL;
+  if (!h->L) return SSHOPM_EUNSUPPORTED;                          // compiled shapes only
+  const int sms = device_sms();
+  if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_classify: no device");
+  long long grid = (N * kmax + 127) / 128;
+  if (grid > (long long)sms * 32) grid = (long long)sms * 32;
+  cudaError_t e = h->L->classify(N, kmax, d_entries, d_count, d_lambda, d_x, ctol, d_out_type, (int)grid,
+                                 (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_classify: launch");
+  h->launches.fetch_add(1);
+  return SSHOPM_OK;
+}
+
 int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x,
                  float* d_out_g, float* d_out_lam, void* stream) {
   if (!h || N < 0) return SSHOPM_EINVAL;

@@ -84,6 +84,12 @@ cudaError_t pack(long long n, const float* e, float4* packed, unsigned int* coun
   return cudaGetLastError();
 }
 
+cudaError_t classify(long long n, int kmax, const float* e, const int32_t* count, const float* lam, const float* x,
+                     float ctol, int8_t* out, int grid, cudaStream_t st) {
+  sshopm_classify_kernel<M, N><<<grid, 128, 0, st>>>(n, kmax, e, count, lam, x, ctol, out);
+  return cudaGetLastError();
+}
+
 cudaError_t apply(long long n_items, const float4* packed, const float* x, float* g, float* lam, int grid, cudaStream_t st) {
   sshopm_apply_kernel<M, N><<<grid, 256, 0, st>>>(n_items, packed, x, g, lam);
   return cudaGetLastError();
@@ -92,7 +98,7 @@ cudaError_t apply(long long n_items, const float4* packed, const float* x, float
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
                       Sh::BFORM ? 1 : 0, 10, 1,
-                      class_index, occupancy, pack, solve, apply};
+                      class_index, occupancy, pack, solve, classify, apply};
 }  // namespace
 
 #define SSHOPM_CAT2(a, b, c) get_launchers_##a##_##b

@@ -711,6 +711,154 @@ sshopm_solve_tpl_kernel(const SolveParams p) {
   }
 }
 
+
+// ---------------------------------------------------------- classify kernel --
+constexpr int pair_row(int pr, int n) { int i = 0; while (pr >= n - i) { pr -= n - i; ++i; } return i; }
+constexpr int pair_col(int pr, int n) { int i = 0; while (pr >= n - i) { pr -= n - i; ++i; } return i + pr; }
+
+// Eigenpair type of each dedup record (reading R18): projected Hessian
+// C = U^T [(m-1) A x^{m-2} - lam I] U on x-perp (Kolda-Mayo second-order test;
+// fibre directions = local maxima).  U = the Householder
+// reflection mapping e_k to x, minus column k.  Eigenvalues of C by cyclic
+// Jacobi.  Codes: +1 max, -1 min, 0 saddle, 2 degenerate (|mu| <= ctol*max(1,|lam|)), 3 empty slot.
+template <int M, int N>
+__global__ void __launch_bounds__(128)
+sshopm_classify_kernel(long long n_tensors, int kmax, const float* __restrict__ entries, const int32_t* __restrict__ count,
+                       const float* __restrict__ lam_in, const float* __restrict__ x_in, float ctol,
+                       int8_t* __restrict__ out) {
+  using T2 = Tables2<M, N>;
+  constexpr T2 T{};
+  constexpr int U = Tables<M, N>::U;
+  for (long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x; idx < n_tensors * kmax;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const long long v = idx / kmax;
+    const int slot = (int)(idx - v * kmax);
+    if (slot >= count[v]) { out[idx] = 3; continue; }
+    float a[U];
+#pragma unroll
+    for (int c = 0; c < U; ++c) a[c] = __ldg(entries + v * U + c);
+    float x[N];
+    float nx = 0.f;
+#pragma unroll
+    for (int j = 0; j < N; ++j) { x[j] = x_in[idx * N + j]; nx = fmaf(x[j], x[j], nx); }
+    const float rx = rsqrtf(nx);
+#pragma unroll
+    for (int j = 0; j < N; ++j) x[j] *= rx;
+    const float lam = lam_in[idx];
+    // H = (m-1) A x^{m-2} - lam I
+    float H[N][N];
+#pragma unroll
+    for (int i = 0; i < N; ++i)
+#pragma unroll
+      for (int j = 0; j < N; ++j) H[i][j] = 0.f;
+    static_for<T2::Q2>([&](auto qq) {
+      constexpr int q = decltype(qq)::value;
+      float mono = (float)T.r_coef[q];
+      static_for<T2::D2>([&](auto tt) {
+        constexpr int t = decltype(tt)::value;
+        constexpr int var = T.r_idx[q][t];
+        mono *= x[var];
+      });
+      static_for<T2::NPR>([&](auto pp) {
+        constexpr int pr = decltype(pp)::value;
+        constexpr int cls = T.r_cls[q][pr];
+        constexpr int i = pair_row(pr, N), j = pair_col(pr, N);
+        H[i][j] = fmaf(mono, a[cls], H[i][j]);
+      });
+    });
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+#pragma unroll
+      for (int j = i; j < N; ++j) {
+        H[i][j] *= (float)(M - 1);
+        H[j][i] = H[i][j];
+      }
+      H[i][i] -= lam;
+    }
+    // Householder P = I - 2 w w^T / (w^T w), w = x + s e_k (s = sign x_k, k = argmax |x_k|): P e_k = -s x
+    int kk = 0;
+#pragma unroll
+    for (int j = 1; j < N; ++j) kk = fabsf(x[j]) > fabsf(x[kk]) ? j : kk;
+    float w[N];
+    float ww = 0.f;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      w[j] = x[j] + ((j == kk) ? (x[kk] >= 0.f ? 1.f : -1.f) : 0.f);
+      ww = fmaf(w[j], w[j], ww);
+    }
+    const float beta = 2.f / ww;
+    // B = P H P = H - beta w (H w)^T - beta (H w) w^T + beta^2 (w^T H w) w w^T
+    float hw[N];
+    float whw = 0.f;
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      float t = 0.f;
+#pragma unroll
+      for (int j = 0; j < N; ++j) t = fmaf(H[i][j], w[j], t);
+      hw[i] = t;
+      whw = fmaf(w[i], t, whw);
+    }
+    constexpr int R = N - 1;
+    float Cm[R > 0 ? R : 1][R > 0 ? R : 1];
+#pragma unroll
+    for (int i = 0; i < R; ++i)
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        const int ii = i + (i >= kk), jj = j + (j >= kk);
+        float hij = 0.f, wi = 0.f, wj = 0.f, hwi = 0.f, hwj = 0.f;
+#pragma unroll
+        for (int r2 = 0; r2 < N; ++r2) {
+          if (r2 == ii) { wi = w[r2]; hwi = hw[r2]; }
+          if (r2 == jj) { wj = w[r2]; hwj = hw[r2]; }
+#pragma unroll
+          for (int c2 = 0; c2 < N; ++c2)
+            if (r2 == ii && c2 == jj) hij = H[r2][c2];
+        }
+        Cm[i][j] = hij - beta * wi * hwj - beta * hwi * wj + beta * beta * whw * wi * wj;
+      }
+    // cyclic Jacobi
+#pragma unroll 1
+    for (int sweep = 0; sweep < 12; ++sweep) {
+#pragma unroll
+      for (int p_ = 0; p_ < R; ++p_)
+#pragma unroll
+        for (int q_ = p_ + 1; q_ < R; ++q_) {
+          const float apq = Cm[p_][q_];
+          if (fabsf(apq) < 1e-30f) continue;
+          const float theta = (Cm[q_][q_] - Cm[p_][p_]) / (2.f * apq);
+          const float t = copysignf(1.f, theta) / (fabsf(theta) + sqrtf(theta * theta + 1.f));
+          const float c = rsqrtf(t * t + 1.f), sn = t * c;
+#pragma unroll
+          for (int r2 = 0; r2 < R; ++r2) {
+            const float crp = Cm[r2][p_], crq = Cm[r2][q_];
+            Cm[r2][p_] = c * crp - sn * crq;
+            Cm[r2][q_] = sn * crp + c * crq;
+          }
+#pragma unroll
+          for (int r2 = 0; r2 < R; ++r2) {
+            const float cpr = Cm[p_][r2], cqr = Cm[q_][r2];
+            Cm[p_][r2] = c * cpr - sn * cqr;
+            Cm[q_][r2] = sn * cpr + c * cqr;
+          }
+        }
+    }
+    const float thr = ctol * fmaxf(1.f, fabsf(lam));
+    int npos = 0, nneg = 0, nzero = 0;
+#pragma unroll
+    for (int i = 0; i < R; ++i) {
+      const float mu = Cm[i][i];
+      nzero += fabsf(mu) <= thr;
+      npos += mu > thr;
+      nneg += mu < -thr;
+    }
+    int8_t code = 0;
+    if (nzero) code = 2;
+    else if (nneg == R) code = 1;
+    else if (npos == R) code = -1;
+    out[idx] = code;
+  }
+}
+
 // ------------------------------------------------------------ apply kernel --
 template <int M, int N>
 __global__ void __launch_bounds__(256)

@@ -130,6 +130,42 @@ struct Tables {
   }
 };
 
+// Degree-(M-2) tables for A x^{M-2} (Definition 2 with p = 2, used by the
+// eigenpair classification): (A x^{M-2})_{ij} = sum_{|r| = M-2} [(M-2)!/r!] a_{class(r + e_i + e_j)} x^r.
+template <int M, int N>
+struct Tables2 {
+  static constexpr int D2 = M - 2;
+  static constexpr int Q2 = binom(D2 + N - 1, D2);     // 1 when M = 2 (the empty monomial)
+  static constexpr int NPR = N * (N + 1) / 2;          // pairs i <= j
+  int r_idx[Q2][D2 > 0 ? D2 : 1];
+  long long r_coef[Q2];
+  int r_cls[Q2][NPR];
+  constexpr Tables2() : r_idx(), r_coef(), r_cls() {
+    int I[M > 2 ? M - 2 : 1] = {};
+    for (int q = 0; q < Q2; ++q) {
+      long long den = 1; int run = 1;
+      for (int t = 0; t < D2; ++t) {
+        r_idx[q][t] = I[t];
+        if (t > 0 && I[t] == I[t - 1]) { ++run; den *= run; } else run = 1;
+      }
+      r_coef[q] = fact(D2) / den;
+      int pr = 0;
+      for (int i = 0; i < N; ++i)
+        for (int j = i; j < N; ++j) {
+          int K[M] = {};
+          int a = 0, b = 0, ins = 0;
+          const int add[2] = {i, j};
+          while (b < M) {                                  // merge the sorted tuple I with (i, j)
+            if (ins < 2 && (a >= D2 || add[ins] <= I[a])) K[b++] = add[ins++];
+            else K[b++] = I[a++];
+          }
+          r_cls[q][pr++] = tuple_rank(K, M, N);
+        }
+      if (D2 > 0) next_tuple(I, D2, N);
+    }
+  }
+};
+
 // Flop counts.
 template <int M, int N>
 constexpr long long paper_flops_per_iter() {

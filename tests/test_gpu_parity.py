@@ -387,3 +387,42 @@ def test_general_kernel_on_compiled_shape(dev):
     both = (a3[3] == 1) & (a1[3] == 1)
     assert both.mean() > 0.5
     assert np.all(np.abs(a3[0][both] - a1[0][both]) <= 1e-4 * np.maximum(1, np.abs(a1[0][both])))
+
+
+# ------------------------------------------------------------ classification --
+@pytest.mark.parametrize("m,n,alpha", [(4, 3, 0.0), (6, 3, 0.25), (4, 6, 0.0), (3, 3, 1.0), (4, 3, -0.5), (8, 3, 0.5)])
+def test_classify_matches_oracle(dev, m, n, alpha):
+    """Reading R18 types of the GPU's dedup records == oracle types of the same records (FP64),
+    except records whose oracle margin min|mu| is within a factor 10 of ctol (borderline)."""
+    from oracle import classify as OC
+    V = 96 if m <= 6 else 24
+    ent = syn.gen_voxels(m, n, 300, V, 5) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 5)
+    st = syn.gen_starts(128, n, 0)
+    s = sh.Solver(m, n)
+    e = torch.from_numpy(ent).to(dev)
+    lam, x, it, cv = s.solve(e, torch.from_numpy(st).to(dev), alpha, 1e-7, 500)
+    cnt, cl, cx, mu, rp = s.dedup(lam, x, cv, 1e-2, 0.05, 6)
+    ctol = 1e-3
+    ty = s.classify(e, cnt, cl, cx, ctol).cpu().numpy()
+    ot, margin = OC.classify(ent, m, n, cnt.cpu().numpy(), cl.cpu().numpy().astype(np.float64),
+                             cx.cpu().numpy().astype(np.float64), ctol)
+    border = (margin > ctol / 10) & (margin < ctol * 10)
+    diff = (ty != ot) & ~border
+    assert not diff.any(), (np.argwhere(diff)[:5], ty[diff][:5], ot[diff][:5])
+    assert set(np.unique(ty)) <= {-1, 0, 1, 2, 3}
+
+
+def test_classify_convex_shift_gives_maxima(dev):
+    """With the automatic convex shift lambda_k only increases, so no local minimum is ever reported; the
+    lambda-stopping rule can stop on the slow ascent past a saddle, so saddles are rare but possible."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, 64, 1)
+    s = sh.Solver(m, n)
+    e = torch.from_numpy(ent).to(dev)
+    lam, x, it, cv = s.solve(e, torch.from_numpy(syn.gen_starts(64, n, 0)).to(dev), "auto_max", 1e-9, 20000)
+    cnt, cl, cx, mu, rp = s.dedup(lam, x, cv, 1e-2, 0.05, 8)
+    ty = s.classify(e, cnt, cl, cx, 1e-3).cpu().numpy()
+    filled = ty != 3
+    assert filled.any()
+    assert not (ty == -1).any()
+    assert np.mean(np.isin(ty[filled], (1, 2))) >= 0.9
