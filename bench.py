@@ -39,7 +39,7 @@ LAM_TOL, ANG_TOL, KMAX = 1e-2, 0.05, 4
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C2", choices=sorted(syn.CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -78,6 +78,18 @@ class ClockSampler:
             self.max_mhz = None
         self._stop = threading.Event()
 
+    def _sample(self):
+        nv = self.nv
+        try:
+            self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+            r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h) if hasattr(nv, "nvmlDeviceGetCurrentClocksEventReasons") \
+                else nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+            for bit, name in self.REASONS.items():
+                if r & bit and name not in ("gpu_idle",):
+                    self.reasons.add(name)
+        except Exception:
+            pass
+
     def _run(self):
         nv = self.nv
         while not self._stop.is_set():
@@ -97,6 +109,11 @@ class ClockSampler:
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
         return self
+
+    def sample_now(self):
+        """Explicit sample from the timing loop (the GPU is busy while the host enqueues ahead)."""
+        if self.ok:
+            self._sample()
 
     def __exit__(self, *a):
         self._stop.set()
@@ -259,6 +276,8 @@ def main():
             flush.zero_()
             e0, e1, e2 = ev[i]
             e0.record(stream)
+            if i % 4 == 2:
+                clk.sample_now()
             run_path(mid_event=e1)
             if not a.unfused:
                 e1.record(stream)
