@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-voxels", type=int, default=0)
     ap.add_argument("--e2e-chunk", type=int, default=0, help="tensors per run_host chunk (0: auto)")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process group backend for N > 1 (gloo: exercise the multi-rank path on one GPU)")
     return ap.parse_args()
 
 
@@ -211,10 +213,14 @@ def main():
     import paper_conf_ipps_ballardkp11_b200 as sh
     from paper_conf_ipps_ballardkp11_b200 import sharding as SH
 
+    local = local % torch.cuda.device_count()           # gloo test runs may share one GPU
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if a.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     m, n, S, Nloc = cfg["m"], cfg["n"], cfg["S"], cfg["N"]
     solver = sh.Solver(m, n)
     U = solver.U
@@ -257,7 +263,13 @@ def main():
             titers.zero_()
         run_path(count_iters)
         if world > 1:
+            gather()
+
+    def gather():
+        if a.backend == "nccl":
             SH.gather_records(rec, rank, world)
+        else:                                             # gloo: stage through host memory
+            SH.gather_records(rec.cpu(), rank, world)
 
     for _ in range(max(a.warmup, 3)):
         step()
@@ -282,7 +294,7 @@ def main():
             if not a.unfused:
                 e1.record(stream)
             if world > 1:
-                SH.gather_records(rec, rank, world)
+                gather()
             e2.record(stream)
         torch.cuda.synchronize()
     if world > 1:
@@ -292,7 +304,8 @@ def main():
     t_step = [e0.elapsed_time(e2) for e0, e1, e2 in ev]
     t_solve = [e0.elapsed_time(e1) for e0, e1, e2 in ev]   # pack + solve kernels (with --solve-dedup: the whole call)
     tot_ms = float(sum(t_step))
-    stats = torch.tensor([tot_ms, float(iters_local), float(sum(t_solve))], dtype=torch.float64, device=dev)
+    cdev = dev if a.backend == "nccl" else torch.device("cpu")
+    stats = torch.tensor([tot_ms, float(iters_local), float(sum(t_solve))], dtype=torch.float64, device=cdev)
     if world > 1:
         tmax = stats[[0, 2]].clone()
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
@@ -322,7 +335,7 @@ def main():
             solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
                             chunk_tensors=chunk, out=outs)
         e2e_s = time.perf_counter() - t0
-        e2e_t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        e2e_t = torch.tensor([e2e_s], dtype=torch.float64, device=dev if a.backend == "nccl" else "cpu")
         if world > 1:
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         e2e_s = float(e2e_t[0])
@@ -370,7 +383,8 @@ def main():
                    "dedup": {"lam_tol": LAM_TOL, "ang_tol": ANG_TOL, "kmax": KMAX},
                    "flop_count": "paper-style F_paper(m,n) x sum(iters), reading R12",
                    "l2": "flushed between timed steps (512 MiB write outside the events)",
-                   "parallelism": f"tensor-range shards x{world}" + (" + NCCL gather of dedup records" if world > 1 else "")},
+                   "parallelism": f"tensor-range shards x{world}" +
+                                  (f" + {a.backend.upper()} gather of dedup records" if world > 1 else "")},
         "voxel_solves_per_s": vps,
         "start_solves_per_s": vps * S,
         "mean_iters": iters_all / (Nloc * world * S),
