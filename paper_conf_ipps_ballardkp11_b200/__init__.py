@@ -133,6 +133,7 @@ class Solver:
         self.paper_flops_per_iter = pf.value
         self.exec_flops_per_iter = ef.value
         self._ws = None            # cached device workspace (torch uint8 tensor)
+        self._ws_size = {}         # (N, S) -> bytes
 
     def close(self):
         if getattr(self, "_h", None):
@@ -151,9 +152,12 @@ class Solver:
         return out
 
     def workspace_size(self, N, S):
-        b = ctypes.c_size_t()
-        _check(lib().sshopm_workspace_size(self._h, int(N), int(S), ctypes.byref(b)), "sshopm_workspace_size")
-        return b.value
+        key = (int(N), int(S))
+        if key not in self._ws_size:
+            b = ctypes.c_size_t()
+            _check(lib().sshopm_workspace_size(self._h, int(N), int(S), ctypes.byref(b)), "sshopm_workspace_size")
+            self._ws_size[key] = b.value
+        return self._ws_size[key]
 
     def _workspace(self, N, S, device):
         need = self.workspace_size(N, S)

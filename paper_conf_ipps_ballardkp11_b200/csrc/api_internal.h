@@ -9,6 +9,9 @@ namespace sshopm { struct HostCache; struct GeneralTables; }
 
 struct sshopm_ctx {
   const sshopm::Launchers* L;      // compiled (m, n) kernels, or null
+  // host-side launch-shape cache (occupancy per non-fused kernel variant, per device); 0 = not computed
+  std::atomic<int> occ_dev;
+  std::atomic<int> occ[4][2][3];   // [shift][wide][schedule]
   sshopm::GeneralTables* gen;      // table-driven kernel tables (any (m, n))
   int m, n, U;
   std::atomic<long long> launches;

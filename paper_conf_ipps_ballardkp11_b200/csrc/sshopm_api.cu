@@ -100,11 +100,34 @@ int release_workspace(Workspace* ws, cudaStream_t st) {
   return SSHOPM_OK;
 }
 
+static std::atomic<int> g_sms_cache[64];
+
 int device_sms() {
   int dev = 0, sms = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) return -1;
+  if (dev >= 0 && dev < 64 && (sms = g_sms_cache[dev].load(std::memory_order_relaxed)) > 0) return sms;
   if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return -1;
+  if (dev >= 0 && dev < 64) g_sms_cache[dev].store(sms, std::memory_order_relaxed);
   return sms;
+}
+
+// occupancy of a non-fused solve variant, cached in the handle for the current device
+static cudaError_t cached_occupancy(sshopm_ctx* h, int shift, bool wide, int schedule, int* bps) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (h->occ_dev.load(std::memory_order_acquire) != dev + 1) {
+    for (auto& a : h->occ)
+      for (auto& b : a)
+        for (auto& c : b) c.store(0, std::memory_order_relaxed);
+    h->occ_dev.store(dev + 1, std::memory_order_release);
+  }
+  std::atomic<int>& slot = h->occ[shift][wide ? 1 : 0][schedule - 1];
+  int v = slot.load(std::memory_order_relaxed);
+  if (v > 0) { *bps = v; return cudaSuccess; }
+  cudaError_t e = h->L->occupancy(shift, wide, schedule, 0, 0, &v);
+  if (e == cudaSuccess && v > 0) slot.store(v, std::memory_order_relaxed);
+  *bps = v;
+  return e;
 }
 }  // namespace sshopm
 
@@ -149,6 +172,10 @@ int sshopm_create(int m, int n, sshopm_t* out) {
   h->U = L ? L->U : gen->U;
   h->launches.store(0);
   h->hc = nullptr;
+  h->occ_dev.store(0);
+  for (auto& a : h->occ)
+    for (auto& b : a)
+      for (auto& c : b) c.store(0);
   *out = h;
   return SSHOPM_OK;
 }
@@ -236,7 +263,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;   // 3 (general) handled above
   if (shift == 3) schedule = 1;                                  // per-tensor alpha: schedule 1 only
   int bps = 0;
-  cudaError_t e = L->occupancy(shift, wide, schedule, 0, 0, &bps);
+  cudaError_t e = cached_occupancy(h, shift, wide, schedule, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
   if (bps < 1) bps = 1;
   // fused dedup (opt-in, opts->fuse_dedup = 1): schedule 1, S <= 1024, and only if its shared memory
