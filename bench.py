@@ -285,11 +285,11 @@ def main():
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
         for i in range(a.steps):
+            if i % 4 == 2:
+                clk.sample_now()                          # host-side NVML query: outside the event window
             flush.zero_()
             e0, e1, e2 = ev[i]
             e0.record(stream)
-            if i % 4 == 2:
-                clk.sample_now()
             run_path(mid_event=e1)
             if not a.unfused:
                 e1.record(stream)
