@@ -361,11 +361,13 @@ def main():
     fmax = pk.get("sm_max_mhz") or clk.max_mhz or 1965.0
     peak_tflops = sms * 128 * 2 * fmax * 1e6 / 1e12
     achieved = Fx * iters_local * a.steps / (solve_ms / 1e3) / 1e12     # rank-local solve kernel
-    traffic = None
+    traffic = fma_pct = None
     tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tf):
         with open(tf) as fh:
-            traffic = json.load(fh).get(a.config)
+            prof = json.load(fh)
+        traffic = prof.get(a.config)
+        fma_pct = prof.get(a.config + "_fma_pipe_active_pct")
     cpu = None
     if world == 1 and not a.no_cpu:
         nv = a.cpu_voxels or (16384 if (m, n) == (4, 3) else 512)
@@ -394,6 +396,7 @@ def main():
                      "kernel": f"sshopm_solve_kernel<{m},{n}>",
                      "peak_basis": f"{sms} SM x 128 FP32 lanes x 2 x {fmax:.0f} MHz (sm_max_mhz)",
                      "flops_per_update": Fx,
+                     "fma_pipe_active_pct_ncu": fma_pct,
                      "flops_note": "algorithmic FP32 flops per (tensor,start,update): monomials + 2*T1 + lambda + shift + norm + scale (DESIGN.md 7)"},
         "cpu_baseline": cpu,
         "e2e": e2e,
