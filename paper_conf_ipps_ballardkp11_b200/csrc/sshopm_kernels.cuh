@@ -279,6 +279,67 @@ __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&
   return lam;
 }
 
+// One SS-HOPM step (Fig. 1) for one lane: lam_k = x_k . A x_k^{m-1}; the stop
+// test (R2, R6, maxit); x_{k+1} = +-(g + alpha x) / ||.|| (lines 2-7, R5).
+// Stopped lanes freeze (x, lambda_prev, k unchanged) so a frozen lane
+// recomputes bit-identical values until the warp refills it.
+// SHIFT: 0 alpha = 0, 1 alpha > 0, 2 alpha < 0 (alpha passed negated), 3 per-lane (la = |alpha|, ls = sign)
+template <int M, int N, int SHIFT>
+__device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[Shape<M, N>::NX], float& lam,
+                                            float& lamp, int& k, bool& conv, bool& stop, bool has, float alpha,
+                                            float la, float ls, float tol, int maxit) {
+  using S = Shape<M, N>;
+  constexpr bool XL = X21<M, N>::v;
+  float2 gp[S::NP > 0 ? S::NP : 1];
+  float gs = 0.f;
+  lam = evaluate<M, N>(cf, xs, gp, gs);                       // g = A x_k^{m-1}, lam_k = x_k . g
+  conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));  // R2 (NaN lamp -> false)
+  // xhat = +-(g + alpha x)   (Fig. 1 lines 2-5, R5)
+  float2 hp[S::NX];
+  static_for<S::NP>([&](auto qq) {
+    constexpr int i = decltype(qq)::value;
+    if constexpr (SHIFT == 0) hp[i] = gp[i];
+    else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
+    else if constexpr (SHIFT == 2) hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
+    else hp[i] = __ffma2_rn(bc(la), xs[i], __fmul2_rn(gp[i], bc(ls)));
+  });
+  if constexpr (S::ODD) {
+    float h;
+    if constexpr (SHIFT == 0) h = gs;
+    else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
+    else if constexpr (SHIFT == 2) h = fmaf(alpha, xs[S::NX - 1].x, -gs);
+    else h = fmaf(la, xs[S::NX - 1].x, gs * ls);
+    hp[S::NX - 1] = f2(h, 0.f);
+  }
+  float nn;
+  {
+    float2 t = __fmul2_rn(hp[0], hp[0]);
+    static_for<S::NX - 1>([&](auto qq) {
+      constexpr int i = decltype(qq)::value + 1;
+      if constexpr (S::ODD && i == S::NX - 1) t.x = fmaf(hp[i].x, hp[i].x, t.x);
+      else t = __ffma2_rn(hp[i], hp[i], t);
+    });
+    nn = t.x + t.y;
+  }
+  const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
+  stop = (!has) | conv | (k >= maxit) | deg;                  // non-short-circuit: one predicate chain
+  const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
+  // the freeze is a guarded update that ptxas if-converts into predicated
+  // FMUL2 / FMUL / MOV / IADD: no select per component (+9% step throughput
+  // on B200, tools/microbench/step_loop.cu)
+  if (!stop) {
+    if constexpr (XL) {
+      xs[0] = __fmul2_rn(hp[0], bc(r));
+      xs[1] = f2(hp[1].x * r, xs[0].y);
+    } else {
+#pragma unroll
+      for (int i = 0; i < S::NX; ++i) xs[i] = __fmul2_rn(hp[i], bc(r));
+    }
+    lamp = lam;
+    ++k;
+  }
+}
+
 // ------------------------------------------------------------ solve kernel --
 struct SolveParams {
   const float4* packed;      // [N][PW/4] from sshopm_pack_kernel
@@ -498,60 +559,9 @@ sshopm_solve_kernel(const SolveParams p) {
 
     // ---------------- SS-HOPM steps (Fig. 1), STEPS per refill check ----------------
 #pragma unroll
-    for (int rep = 0; rep < STEPS; ++rep) {
-      float2 gp[S::NP > 0 ? S::NP : 1];
-      float gs = 0.f;
-      lam = evaluate<M, N>(cf, xs, gp, gs);                       // g = A x_k^{m-1}, lam_k = x_k . g
-      conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));  // R2 (NaN lamp -> false)
-      // xhat = +-(g + alpha x)   (Fig. 1 lines 2-5, R5)
-      float2 hp[S::NX];
-      static_for<S::NP>([&](auto qq) {
-        constexpr int i = decltype(qq)::value;
-        if constexpr (SHIFT == 0) hp[i] = gp[i];
-        else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
-        else if constexpr (SHIFT == 2) hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
-        else hp[i] = __ffma2_rn(bc(la), xs[i], __fmul2_rn(gp[i], bc(ls)));
-      });
-      if constexpr (S::ODD) {
-        float h;
-        if constexpr (SHIFT == 0) h = gs;
-        else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
-        else if constexpr (SHIFT == 2) h = fmaf(alpha, xs[S::NX - 1].x, -gs);
-        else h = fmaf(la, xs[S::NX - 1].x, gs * ls);
-        hp[S::NX - 1] = f2(h, 0.f);
-      }
-      float nn;
-      {
-        float2 t = __fmul2_rn(hp[0], hp[0]);
-        static_for<S::NX - 1>([&](auto qq) {
-          constexpr int i = decltype(qq)::value + 1;
-          if constexpr (S::ODD && i == S::NX - 1) t.x = fmaf(hp[i].x, hp[i].x, t.x);
-          else t = __ffma2_rn(hp[i], hp[i], t);
-        });
-        nn = t.x + t.y;
-      }
-      const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
-      stop = !has || conv || k >= maxit || deg;
-      const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
-      // freeze stopped lanes by selection (no branch): x, lambda_prev, k keep their values
-      if constexpr (XL) {
-        const float2 n01 = __fmul2_rn(hp[0], bc(r));
-        const float n2 = hp[1].x * r;
-        xs[0].x = stop ? xs[0].x : n01.x;
-        xs[0].y = stop ? xs[0].y : n01.y;
-        xs[1].x = stop ? xs[1].x : n2;
-        xs[1].y = xs[0].y;
-      } else {
-#pragma unroll
-        for (int i = 0; i < S::NX; ++i) {
-          const float2 nx = __fmul2_rn(hp[i], bc(r));
-          xs[i].x = stop ? xs[i].x : nx.x;
-          xs[i].y = stop ? xs[i].y : nx.y;
-        }
-      }
-      lamp = stop ? lamp : lam;
-      k += stop ? 0 : 1;
-    }
+    for (int rep = 0; rep < STEPS; ++rep)
+      sshopm_step<M, N, SHIFT>(cf, xs, lam, lamp, k, conv, stop, has, alpha, la, ls, tol, maxit);
+    __syncwarp();
   }
 
   if (p.total_iters) {
@@ -652,56 +662,8 @@ sshopm_solve_tpl_kernel(const SolveParams p) {
     }
 
 #pragma unroll
-    for (int rep = 0; rep < STEPS; ++rep) {
-      float2 gp[S::NP > 0 ? S::NP : 1];
-      float gs = 0.f;
-      lam = evaluate<M, N>(cf, xs, gp, gs);
-      conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
-      float2 hp[S::NX];
-      static_for<S::NP>([&](auto qq) {
-        constexpr int i = decltype(qq)::value;
-        if constexpr (SHIFT == 0) hp[i] = gp[i];
-        else if constexpr (SHIFT == 1) hp[i] = __ffma2_rn(bc(alpha), xs[i], gp[i]);
-        else hp[i] = __ffma2_rn(bc(alpha), xs[i], f2(-gp[i].x, -gp[i].y));
-      });
-      if constexpr (S::ODD) {
-        float h;
-        if constexpr (SHIFT == 0) h = gs;
-        else if constexpr (SHIFT == 1) h = fmaf(alpha, xs[S::NX - 1].x, gs);
-        else h = fmaf(alpha, xs[S::NX - 1].x, -gs);
-        hp[S::NX - 1] = f2(h, 0.f);
-      }
-      float nn;
-      {
-        float2 q = __fmul2_rn(hp[0], hp[0]);
-        static_for<S::NX - 1>([&](auto qq) {
-          constexpr int i = decltype(qq)::value + 1;
-          if constexpr (S::ODD && i == S::NX - 1) q.x = fmaf(hp[i].x, hp[i].x, q.x);
-          else q = __ffma2_rn(hp[i], hp[i], q);
-        });
-        nn = q.x + q.y;
-      }
-      const bool deg = !(nn >= 1.17549435e-38f);
-      stop = !has || conv || k >= maxit || deg;
-      const float r = rsqrt_ftz(nn);
-      if constexpr (XL) {
-        const float2 n01 = __fmul2_rn(hp[0], bc(r));
-        const float n2 = hp[1].x * r;
-        xs[0].x = stop ? xs[0].x : n01.x;
-        xs[0].y = stop ? xs[0].y : n01.y;
-        xs[1].x = stop ? xs[1].x : n2;
-        xs[1].y = xs[0].y;
-      } else {
-#pragma unroll
-        for (int i = 0; i < S::NX; ++i) {
-          const float2 nx = __fmul2_rn(hp[i], bc(r));
-          xs[i].x = stop ? xs[i].x : nx.x;
-          xs[i].y = stop ? xs[i].y : nx.y;
-        }
-      }
-      lamp = stop ? lamp : lam;
-      k += stop ? 0 : 1;
-    }
+    for (int rep = 0; rep < STEPS; ++rep)
+      sshopm_step<M, N, SHIFT>(cf, xs, lam, lamp, k, conv, stop, has, alpha, 0.f, 1.f, tol, maxit);
   }
 
   if (p.total_iters) {
