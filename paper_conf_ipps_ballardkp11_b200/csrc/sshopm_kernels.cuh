@@ -45,9 +45,18 @@ __device__ __forceinline__ float2 bc(float a) { return make_float2(a, a); }
 __device__ __forceinline__ float4 ldg4(const float4* p) { return __ldg(p); }
 
 constexpr int round4(int v) { return (v + 3) / 4 * 4; }
-#ifndef SSHOPM_STEPS
-#define SSHOPM_STEPS 2
+// SS-HOPM steps per refill check (trip).  More steps amortise the ballot and
+// branch over more arithmetic but let stopped lanes idle longer; measured on
+// B200 (C2, (4,3)): 1 step 4.90 ms, 2 steps 4.60, 3 steps 4.45, 4 steps 4.58
+// (best refill threshold each).  Shapes with costlier steps keep 2.
+template <int M, int N>
+constexpr int steps_per_trip() {
+#ifdef SSHOPM_STEPS
+  return SSHOPM_STEPS;
+#else
+  return (binom(M + N - 2, M - 1) * N <= 30) ? 3 : 2;
 #endif
+}
 
 template <int M, int N>
 struct Shape {
@@ -387,7 +396,7 @@ template <int M, int N, int SHIFT, bool WIDE, int FUSED_MODE>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
   constexpr bool FUSED = FUSED_MODE != 0;        // 1: shared-memory dedup (any S <= 1024), 2: register dedup (S = 128)
-  constexpr int STEPS = SSHOPM_STEPS;        // SS-HOPM steps between refill checks
+  constexpr int STEPS = steps_per_trip<M, N>();        // SS-HOPM steps between refill checks
   using S = Shape<M, N>;
   using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
   constexpr int SST4 = round4(N) / 4;
@@ -432,13 +441,16 @@ sshopm_solve_kernel(const SolveParams p) {
   bool has = false, stop = true, conv = false;
   Idx item = 0;
   float la = 0.f, ls = 1.f;  // SHIFT == 3: per-lane |alpha| and sign: xhat = ls*g + la*x
-  unsigned long long it_sum = 0;
+  uint32_t it_sum = 0;       // per-lane sum of iterations (<= items per lane x maxit; flushed as 64-bit)
+  // refill threshold: K idle lanes while items remain, all 32 once the chunks are exhausted,
+  // so the per-trip check is one ballot, one popc and one compare (K in [1, 32], host-clamped)
+  uint32_t k_eff = (uint32_t)p.refill_k;
 
   for (;;) {
     // ---------------- refill (warp-uniform branch) ----------------
     const uint32_t smask = __ballot_sync(FULL, stop);
     const uint32_t cnt = __popc(smask);
-    if ((cnt >= (uint32_t)p.refill_k && !exhausted) || smask == FULL) {
+    if (cnt >= k_eff) {
       // straight-line refill: predicated stores / loads, selects for state (no divergent regions)
       const uint32_t avail = c_end - c_next;                 // invariant: c_next <= c_end
       uint32_t n_end = 0;
@@ -473,7 +485,7 @@ sshopm_solve_kernel(const SolveParams p) {
         p.out_iters[item] = k;
         p.out_conv[item] = conv ? 1 : 0;
       }
-      it_sum += wr ? (unsigned long long)k : 0ull;
+      it_sum += wr ? (uint32_t)k : 0u;
       bool chunk_done = false;
       int done_slot = 0;                                   // ring slot of the chunk this lane completed
       if constexpr (FUSED) {
@@ -514,7 +526,7 @@ sshopm_solve_kernel(const SolveParams p) {
       has = stop ? ok : has;
       if (!exhausted) {
         if (cnt > avail) {
-          if (n_end == 0) exhausted = true;
+          if (n_end == 0) { exhausted = true; k_eff = 32u; }
           c_vox = n_vox;
           c_next = min(cnt - avail, n_end);                // a chunk smaller than the request is used up
           c_end = n_end;
@@ -565,9 +577,10 @@ sshopm_solve_kernel(const SolveParams p) {
   }
 
   if (p.total_iters) {
+    unsigned long long ws = it_sum;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) it_sum += __shfl_xor_sync(0xffffffffu, it_sum, o);
-    if (lane == 0) atomicAdd(p.total_iters, it_sum);
+    for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(0xffffffffu, ws, o);
+    if (lane == 0) atomicAdd(p.total_iters, ws);
   }
 }
 
@@ -582,7 +595,7 @@ sshopm_solve_kernel(const SolveParams p) {
 template <int M, int N, int SHIFT, bool WIDE>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_tpl_kernel(const SolveParams p) {
-  constexpr int STEPS = SSHOPM_STEPS;
+  constexpr int STEPS = steps_per_trip<M, N>();
   using S = Shape<M, N>;
   using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
   constexpr int SST4 = round4(N) / 4;

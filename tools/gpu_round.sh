@@ -15,4 +15,6 @@ if [ -z "${SKIP_NCU:-}" ]; then
       python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu "$@" > $OUT/ncu_launch_bench.log 2>&1; echo "ncu launches rc=$?"
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:sshopm_solve -s 3 -c 1 \
       -o $OUT/prof_solve python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu "$@" > $OUT/ncu_full.log 2>&1; echo "ncu full rc=$?"
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:sshopm_dedup -s 3 -c 1 \
+      -o $OUT/prof_dedup python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu "$@" > $OUT/ncu_dedup.log 2>&1; echo "ncu dedup rc=$?"
 fi
