@@ -465,7 +465,7 @@ int make_dedup_params(int n, int64_t N, int S, float lam_tol, float ang_tol, int
 static int dedup_launch_shape(int n, int64_t N, int S, bool fast, int* grid, int* block, int* smem) {
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_dedup: no device");
-  const int per_warp = fast ? 128 * (n + 3) * 4 : dedup_smem_words(S, n) * 4;
+  const int per_warp = fast ? dedup128_smem_per_warp(n) : dedup_smem_words(S, n) * 4;
   int wpb = (96 * 1024) / per_warp;
   if (wpb > 8) wpb = 8;
   if (wpb < 1) wpb = 1;

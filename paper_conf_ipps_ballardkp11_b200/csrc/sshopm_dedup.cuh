@@ -37,10 +37,41 @@ struct DedupParams {
 // shared-memory words per warp for S starts, dimension n
 __host__ __device__ constexpr int dedup_smem_words(int S, int n) { return S * (n + 2) + 3 * S; }
 
-// One warp clusters tensor v (R16).  Staging arrays (per warp, shared memory):
-// s_lam[S], s_x[S*N], s_cid[S], c_lam[S], c_rep[S], c_mult[S].  Inputs are read
-// with ld.global.cg (L2), so the routine is also safe right after other lanes
-// of the same warp wrote them (fused solve -> dedup; caller fences).
+// R16 membership test of a start (ls, xs, squared norm n2s) against the round's
+// representative (rl, rx, squared norm rn), ltol = lam_tol * max(1, |rl|),
+// lim2 = cos_tol^2 * rn.  angle(xs, rx) <= ang_tol is cos >= cos_tol; for
+// ang_tol <= pi/2 (cos_tol >= 0) it is evaluated squared, dot^2 >= lim2 * n2s,
+// with the sign of dot chosen by the R15 rules (no square root); for larger
+// ang_tol as |dot| >= cos_tol * sqrt(n2s * rn).  Every dedup path (standalone,
+// list, fused) calls this one function, so they agree bit for bit.
+template <int N, bool EVEN>
+__device__ __forceinline__ bool dd_same(float ls, const float (&xs)[N], float n2s, float rl, const float (&rx)[N],
+                                        float rn, float lim2, float ltol, float cos_tol) {
+  float dot = 0.f;
+#pragma unroll
+  for (int j = 0; j < N; ++j) dot = fmaf(xs[j], rx[j], dot);
+  if (cos_tol >= 0.f) {   // branch-free (bitwise & / |): predicate logic, no per-start branches
+    const bool ang = dot * dot >= lim2 * n2s;
+    if (EVEN) return ang & (fabsf(ls - rl) <= ltol);
+    return ang & (((dot >= 0.f) & (fabsf(ls - rl) <= ltol)) | ((dot <= 0.f) & (fabsf(-ls - rl) <= ltol)));
+  }
+  const float lim = cos_tol * sqrtf(n2s * rn);
+  if (EVEN) return fabsf(ls - rl) <= ltol && fabsf(dot) >= lim;
+  return (fabsf(ls - rl) <= ltol && dot >= lim) || (fabsf(-ls - rl) <= ltol && -dot >= lim);
+}
+
+template <int N>
+__device__ __forceinline__ float dd_norm2(const float (&x)[N]) {
+  float n2 = 0.f;
+#pragma unroll
+  for (int j = 0; j < N; ++j) n2 = fmaf(x[j], x[j], n2);
+  return n2;
+}
+
+// One warp clusters tensor v (R16), any S.  Staging arrays (per warp, shared
+// memory): s_lam[S], s_x[S*N], s_cid[S], c_lam[S], c_rep[S], c_mult[S].  Inputs
+// are read with ld.global.cg (L2), so the routine is also safe right after
+// other lanes of the same warp wrote them (fused solve -> dedup; caller fences).
 template <int N, bool EVEN>
 __device__ __forceinline__ void warp_dedup_tensor(const DedupParams& p, long long v, int lane, float* s_lam,
                                                   float* s_x, int* s_cid, float* c_lam, int* c_rep, int* c_mult) {
@@ -53,6 +84,7 @@ __device__ __forceinline__ void warp_dedup_tensor(const DedupParams& p, long lon
   for (int t = lane; t < S * N; t += 32) s_x[t] = __ldcg(p.x + b * N + t);
   __syncwarp();
 
+  const float ct2 = p.cos_tol * p.cos_tol;
   int ncl = 0;
   for (;;) {
     int first = 0x7fffffff;
@@ -62,23 +94,18 @@ __device__ __forceinline__ void warp_dedup_tensor(const DedupParams& p, long lon
     if (first == 0x7fffffff) break;
     const float rl = s_lam[first];
     float rx[N];
-    float rn = 0.f;
 #pragma unroll
-    for (int j = 0; j < N; ++j) { rx[j] = s_x[first * N + j]; rn = fmaf(rx[j], rx[j], rn); }
+    for (int j = 0; j < N; ++j) rx[j] = s_x[first * N + j];
+    const float rn = dd_norm2<N>(rx);
     const float ltol = p.lam_tol * fmaxf(1.0f, fabsf(rl));
+    const float lim2 = ct2 * rn;
     int cnt = 0;
     for (int s = lane; s < S; s += 32) {
       if (s_cid[s] != -1) continue;
-      bool same = (s == first);
-      if (!same) {
-        const float ls = s_lam[s];
-        float dot = 0.f, n2 = 0.f;
+      float xs[N];
 #pragma unroll
-        for (int j = 0; j < N; ++j) { const float xv = s_x[s * N + j]; dot = fmaf(xv, rx[j], dot); n2 = fmaf(xv, xv, n2); }
-        const float lim = p.cos_tol * sqrtf(n2 * rn);
-        if (EVEN) same = fabsf(ls - rl) <= ltol && fabsf(dot) >= lim;
-        else same = (fabsf(ls - rl) <= ltol && dot >= lim) || (fabsf(-ls - rl) <= ltol && -dot >= lim);
-      }
+      for (int j = 0; j < N; ++j) xs[j] = s_x[s * N + j];
+      const bool same = (s == first) || dd_same<N, EVEN>(s_lam[s], xs, dd_norm2<N>(xs), rl, rx, rn, lim2, ltol, p.cos_tol);
       if (same) { s_cid[s] = ncl; ++cnt; }
     }
     cnt = __reduce_add_sync(0xffffffffu, cnt);
@@ -157,10 +184,12 @@ __global__ void __launch_bounds__(256) sshopm_dedup_list_kernel(const DedupParam
 }
 
 // ----------------------------------------------------------------------------
-// Fast path for S = 128: lane l owns starts 4l..4l+3 in registers, loaded as
-// float4 (lambda: 1, x: N, converged: one u32), and the next tensor is
-// prefetched while the current one is clustered.  Same rounds as above (round
-// representative = first unassigned converged start in start order).
+// S = 128: lane l owns starts 4l..4l+3 in registers (float4 loads: lambda 1, x N,
+// converged one u32); the unassigned converged starts of a lane are a 4-bit
+// mask; cluster c's record lives in lane c's registers (up to 32 clusters).
+// Same rounds as warp_dedup_tensor.  STAGE: the round representative is read
+// back from a per-warp shared-memory copy of the tensor's results (4 LDS)
+// instead of selected and shuffled out of the owning lane's registers.
 template <int N>
 struct DedupRegs {
   float4 lam;
@@ -169,139 +198,54 @@ struct DedupRegs {
 };
 
 template <int N>
-__device__ __forceinline__ void dedup_load(DedupRegs<N>& r, const DedupParams& p, long long v, int lane) {
+__device__ __forceinline__ void dedup_load(DedupRegs<N>& r, const DedupParams& p, long long v, int lane, bool stream) {
   const long long b = v * 128;
-  r.lam = __ldcs(reinterpret_cast<const float4*>(p.lambda + b) + lane);
+  const float4* pl = reinterpret_cast<const float4*>(p.lambda + b) + lane;
+  const float4* px = reinterpret_cast<const float4*>(p.x + b * N) + lane * N;
+  const unsigned int* pc = reinterpret_cast<const unsigned int*>(p.conv + b) + lane;
+  if (stream) {                    // standalone kernel: read once, evict first
+    r.lam = __ldcs(pl);
 #pragma unroll
-  for (int i = 0; i < N; ++i) r.x[i] = __ldcs(reinterpret_cast<const float4*>(p.x + b * N) + lane * N + i);
-  r.conv = __ldcs(reinterpret_cast<const unsigned int*>(p.conv + b) + lane);
-}
-
-template <int N>
-__device__ __forceinline__ float xcomp(const DedupRegs<N>& r, int c, int j) {   // component j of local start c (c, j compile-time)
-  const int w = c * N + j;
-  const float4 q = r.x[w / 4];
-  return (w % 4 == 0) ? q.x : (w % 4 == 1) ? q.y : (w % 4 == 2) ? q.z : q.w;
-}
-
-template <int N, bool EVEN>
-__global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams p) {
-  constexpr int S = 128, SPL = 4;
-  extern __shared__ float smem[];
-  const int lane = threadIdx.x & 31;
-  const int wib = threadIdx.x >> 5;
-  // per-warp cluster records: lam[S], rep[S], mult[S], x[S][N]
-  float* c_lam = smem + (size_t)wib * S * (N + 3);
-  int* c_rep = reinterpret_cast<int*>(c_lam + S);
-  int* c_mult = c_rep + S;
-  float* c_x = reinterpret_cast<float*>(c_mult + S);
-
-  const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
-  long long v = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
-  DedupRegs<N> nx;
-  if (v < p.n_tensors) dedup_load<N>(nx, p, v, lane);
-  for (; v < p.n_tensors; v += warps) {
-    const DedupRegs<N> cur = nx;
-    if (v + warps < p.n_tensors) dedup_load<N>(nx, p, v + warps, lane);   // prefetch
-    const float lam[SPL] = {cur.lam.x, cur.lam.y, cur.lam.z, cur.lam.w};
-    // cid: -1 unassigned converged, -2 not converged, >= 0 cluster
-    int cid[SPL];
+    for (int i = 0; i < N; ++i) r.x[i] = __ldcs(px + i);
+    r.conv = __ldcs(pc);
+  } else {                         // fused: just written by this warp's lanes, read through L2
+    r.lam = __ldcg(pl);
 #pragma unroll
-    for (int c = 0; c < SPL; ++c) cid[c] = ((cur.conv >> (8 * c)) & 0xffu) ? -1 : -2;
-    int ncl = 0;
-    for (;;) {
-      int first = 0x7fffffff;
-#pragma unroll
-      for (int c = SPL - 1; c >= 0; --c)
-        if (cid[c] == -1) first = SPL * lane + c;
-      first = __reduce_min_sync(0xffffffffu, first);
-      if (first == 0x7fffffff) break;
-      const int src = first / SPL, fc = first % SPL;
-      float rl = (fc == 0) ? lam[0] : (fc == 1) ? lam[1] : (fc == 2) ? lam[2] : lam[3];
-      rl = __shfl_sync(0xffffffffu, rl, src);
-      float rx[N];
-      float rn = 0.f;
-#pragma unroll
-      for (int j = 0; j < N; ++j) {
-        float t = (fc == 0) ? xcomp<N>(cur, 0, j) : (fc == 1) ? xcomp<N>(cur, 1, j) : (fc == 2) ? xcomp<N>(cur, 2, j) : xcomp<N>(cur, 3, j);
-        rx[j] = __shfl_sync(0xffffffffu, t, src);
-        rn = fmaf(rx[j], rx[j], rn);
-      }
-      const float ltol = p.lam_tol * fmaxf(1.0f, fabsf(rl));
-      int cnt = 0;
-#pragma unroll
-      for (int c = 0; c < SPL; ++c) {
-        if (cid[c] != -1) continue;
-        bool same = (SPL * lane + c == first);
-        if (!same) {
-          float dot = 0.f, n2 = 0.f;
-#pragma unroll
-          for (int j = 0; j < N; ++j) { const float xv = xcomp<N>(cur, c, j); dot = fmaf(xv, rx[j], dot); n2 = fmaf(xv, xv, n2); }
-          const float lim = p.cos_tol * sqrtf(n2 * rn);
-          if (EVEN) same = fabsf(lam[c] - rl) <= ltol && fabsf(dot) >= lim;
-          else same = (fabsf(lam[c] - rl) <= ltol && dot >= lim) || (fabsf(-lam[c] - rl) <= ltol && -dot >= lim);
-        }
-        if (same) { cid[c] = ncl; ++cnt; }
-      }
-      cnt = __reduce_add_sync(0xffffffffu, cnt);
-      if (lane == 0) {
-        c_lam[ncl] = rl; c_rep[ncl] = first; c_mult[ncl] = cnt;
-#pragma unroll
-        for (int j = 0; j < N; ++j) c_x[ncl * N + j] = rx[j];
-      }
-      ++ncl;
-    }
-    __syncwarp();
-    if (lane == 0) p.out_count[v] = ncl;
-    const long long ob = v * p.kmax;
-    for (int c = lane; c < ncl; c += 32) {
-      const float lc = c_lam[c];
-      int rank = 0;
-      for (int d = 0; d < ncl; ++d) {
-        const float ld = c_lam[d];
-        rank += (ld > lc) || (ld == lc && d < c);
-      }
-      if (rank < p.kmax) {
-        p.out_lambda[ob + rank] = lc;
-#pragma unroll
-        for (int j = 0; j < N; ++j) p.out_x[(ob + rank) * N + j] = c_x[c * N + j];
-        p.out_mult[ob + rank] = c_mult[c];
-        if (p.out_rep) p.out_rep[ob + rank] = c_rep[c];
-      }
-    }
-    for (int slot = ncl + lane; slot < p.kmax; slot += 32) {
-      p.out_lambda[ob + slot] = 0.f;
-#pragma unroll
-      for (int j = 0; j < N; ++j) p.out_x[(ob + slot) * N + j] = 0.f;
-      p.out_mult[ob + slot] = 0;
-      if (p.out_rep) p.out_rep[ob + slot] = -1;
-    }
-    __syncwarp();
+    for (int i = 0; i < N; ++i) r.x[i] = __ldcg(px + i);
+    r.conv = __ldcg(pc);
   }
 }
 
-// Register-resident clustering of tensor v for S = 128 (fused solve -> dedup):
-// lane l owns starts 4l..4l+3 (float4 loads through L2), cluster c's record
-// lives in lane c's registers.  Returns false (nothing written) if the tensor
-// has more than 32 clusters; the caller then hands it to the list kernel.
-template <int N, bool EVEN>
-__device__ __forceinline__ bool warp_dedup128_regs(const DedupParams& p, long long v, int lane) {
+// Returns false (nothing written) if the tensor has more than 32 clusters.
+// stage: per-warp 128 * (N + 1) floats of shared memory when STAGE.
+template <int N, bool EVEN, bool STAGE>
+__device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v, int lane, const DedupRegs<N>& r,
+                                              float* stage) {
   constexpr int SPL = 4;
-  const long long b = v * 128;
-  const float4 l4 = __ldcg(reinterpret_cast<const float4*>(p.lambda + b) + lane);
-  float4 x4[N];
+  const uint32_t FULL = 0xffffffffu;
+  const float lam[SPL] = {r.lam.x, r.lam.y, r.lam.z, r.lam.w};
+  float xs[SPL][N];
 #pragma unroll
-  for (int i = 0; i < N; ++i) x4[i] = __ldcg(reinterpret_cast<const float4*>(p.x + b * N) + lane * N + i);
-  const uint32_t cv4 = __ldcg(reinterpret_cast<const unsigned int*>(p.conv + b) + lane);
-  const float lam[SPL] = {l4.x, l4.y, l4.z, l4.w};
-  auto xc = [&](int c, int j) -> float {
-    const int w = c * N + j;
-    const float4 q = x4[w / 4];
-    return (w % 4 == 0) ? q.x : (w % 4 == 1) ? q.y : (w % 4 == 2) ? q.z : q.w;
-  };
-  int cid[SPL];
+  for (int c = 0; c < SPL; ++c)
 #pragma unroll
-  for (int c = 0; c < SPL; ++c) cid[c] = ((cv4 >> (8 * c)) & 0xffu) ? -1 : -2;
+    for (int j = 0; j < N; ++j) {
+      const int w = c * N + j;
+      const float4 q = r.x[w / 4];
+      xs[c][j] = (w % 4 == 0) ? q.x : (w % 4 == 1) ? q.y : (w % 4 == 2) ? q.z : q.w;
+    }
+  float n2[SPL];
+#pragma unroll
+  for (int c = 0; c < SPL; ++c) n2[c] = dd_norm2<N>(xs[c]);
+  uint32_t un = 0;                                   // unassigned converged starts (bit c = start 4*lane + c)
+#pragma unroll
+  for (int c = 0; c < SPL; ++c) un |= ((r.conv >> (8 * c)) & 0xffu) ? (1u << c) : 0u;
+  if constexpr (STAGE) {
+    reinterpret_cast<float4*>(stage)[lane] = r.lam;
+#pragma unroll
+    for (int i = 0; i < N; ++i) reinterpret_cast<float4*>(stage + 128)[lane * N + i] = r.x[i];
+    __syncwarp();
+  }
+  const float ct2 = p.cos_tol * p.cos_tol;
   float my_lam = 0.f, my_x[N];
   int my_rep = -1, my_mult = 0;
 #pragma unroll
@@ -309,41 +253,35 @@ __device__ __forceinline__ bool warp_dedup128_regs(const DedupParams& p, long lo
   int ncl = 0;
 #pragma unroll 1
   for (;;) {
-    int first = 0x7fffffff;
-#pragma unroll
-    for (int c = SPL - 1; c >= 0; --c)
-      if (cid[c] == -1) first = SPL * lane + c;
-    first = __reduce_min_sync(0xffffffffu, first);
+    const int fl = __ffs(un) - 1;                    // lowest unassigned local start (-1: none)
+    const int first = __reduce_min_sync(FULL, fl >= 0 ? SPL * lane + fl : 0x7fffffff);
     if (first == 0x7fffffff) break;
-    if (ncl == 32) return false;                      // too many clusters for the register form
-    const int src = first / SPL, fc = first % SPL;
-    float rl = (fc == 0) ? lam[0] : (fc == 1) ? lam[1] : (fc == 2) ? lam[2] : lam[3];
-    rl = __shfl_sync(0xffffffffu, rl, src);
-    float rx[N];
-    float rn = 0.f;
+    if (ncl == 32) return false;                     // too many clusters for the register form
+    float rl, rx[N];
+    if constexpr (STAGE) {
+      rl = stage[first];
 #pragma unroll
-    for (int j = 0; j < N; ++j) {
-      const float t = (fc == 0) ? xc(0, j) : (fc == 1) ? xc(1, j) : (fc == 2) ? xc(2, j) : xc(3, j);
-      rx[j] = __shfl_sync(0xffffffffu, t, src);
-      rn = fmaf(rx[j], rx[j], rn);
+      for (int j = 0; j < N; ++j) rx[j] = stage[128 + first * N + j];
+    } else {
+      const int src = first / SPL, fc = first % SPL;
+      rl = __shfl_sync(FULL, (fc == 0) ? lam[0] : (fc == 1) ? lam[1] : (fc == 2) ? lam[2] : lam[3], src);
+#pragma unroll
+      for (int j = 0; j < N; ++j)
+        rx[j] = __shfl_sync(FULL, (fc == 0) ? xs[0][j] : (fc == 1) ? xs[1][j] : (fc == 2) ? xs[2][j] : xs[3][j], src);
     }
+    const float rn = dd_norm2<N>(rx);
     const float ltol = p.lam_tol * fmaxf(1.0f, fabsf(rl));
-    int cnt = 0;
+    const float lim2 = ct2 * rn;
+    const int fsel = first - SPL * lane;             // local index of the representative if this lane owns it
+    uint32_t hit = 0;
 #pragma unroll
-    for (int c = 0; c < SPL; ++c) {
-      if (cid[c] != -1) continue;
-      bool same = (SPL * lane + c == first);
-      if (!same) {
-        float dot = 0.f, n2 = 0.f;
-#pragma unroll
-        for (int j = 0; j < N; ++j) { const float xv = xc(c, j); dot = fmaf(xv, rx[j], dot); n2 = fmaf(xv, xv, n2); }
-        const float lim = p.cos_tol * sqrtf(n2 * rn);
-        if (EVEN) same = fabsf(lam[c] - rl) <= ltol && fabsf(dot) >= lim;
-        else same = (fabsf(lam[c] - rl) <= ltol && dot >= lim) || (fabsf(-lam[c] - rl) <= ltol && -dot >= lim);
-      }
-      if (same) { cid[c] = ncl; ++cnt; }
+    for (int c = 0; c < SPL; ++c) {                  // evaluated for every start, masked afterwards (no branches)
+      const bool same = (fsel == c) | dd_same<N, EVEN>(lam[c], xs[c], n2[c], rl, rx, rn, lim2, ltol, p.cos_tol);
+      hit |= same ? (1u << c) : 0u;
     }
-    cnt = __reduce_add_sync(0xffffffffu, cnt);
+    hit &= un;
+    un &= ~hit;
+    const int cnt = __reduce_add_sync(FULL, __popc(hit));
     if (lane == ncl) {
       my_lam = rl; my_rep = first; my_mult = cnt;
 #pragma unroll
@@ -355,7 +293,7 @@ __device__ __forceinline__ bool warp_dedup128_regs(const DedupParams& p, long lo
   int rank = 0;
 #pragma unroll 1
   for (int d = 0; d < ncl; ++d) {
-    const float ld = __shfl_sync(0xffffffffu, my_lam, d);
+    const float ld = __shfl_sync(FULL, my_lam, d);
     rank += (ld > my_lam) || (ld == my_lam && d < lane);
   }
   if (lane == 0) p.out_count[v] = ncl;
@@ -375,7 +313,48 @@ __device__ __forceinline__ bool warp_dedup128_regs(const DedupParams& p, long lo
     p.out_mult[ob + slot] = 0;
     if (p.out_rep) p.out_rep[ob + slot] = -1;
   }
+  if constexpr (STAGE) __syncwarp();                 // the stage is rewritten by the next tensor
   return true;
+}
+
+// Standalone dedup for S = 128: warp per tensor, the next tensor prefetched
+// into registers while the current one is clustered; a tensor with more than
+// 32 clusters falls back to the shared-memory routine.
+template <int N, bool EVEN>
+__global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams p) {
+  extern __shared__ float smem[];
+  const int lane = threadIdx.x & 31;
+  const int wib = threadIdx.x >> 5;
+  float* stage = smem + (size_t)wib * 128 * (N + 1);
+  float* gen = smem + (size_t)(blockDim.x >> 5) * 128 * (N + 1) + (size_t)wib * dedup_smem_words(128, N);
+  const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
+  long long v = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
+  DedupRegs<N> nx;
+  if (v < p.n_tensors) dedup_load<N>(nx, p, v, lane, true);
+  for (; v < p.n_tensors; v += warps) {
+    const DedupRegs<N> cur = nx;
+    if (v + warps < p.n_tensors) dedup_load<N>(nx, p, v + warps, lane, true);   // prefetch
+    if (!dedup128_regs<N, EVEN, true>(p, v, lane, cur, stage)) {
+      float* s_lam = gen;
+      float* s_x = s_lam + 128;
+      int* s_cid = reinterpret_cast<int*>(s_x + 128 * N);
+      float* c_lam = reinterpret_cast<float*>(s_cid + 128);
+      int* c_rep = reinterpret_cast<int*>(c_lam + 128);
+      int* c_mult = c_rep + 128;
+      warp_dedup_tensor<N, EVEN>(p, v, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
+    }
+  }
+}
+// shared-memory bytes per warp of sshopm_dedup128_kernel (stage + fallback staging)
+__host__ __device__ constexpr int dedup128_smem_per_warp(int n) { return (128 * (n + 1) + dedup_smem_words(128, n)) * 4; }
+
+// Register-resident clustering of tensor v for S = 128 inside the solve kernel
+// (fused solve -> dedup, no staging shared memory).
+template <int N, bool EVEN>
+__device__ __forceinline__ bool warp_dedup128_regs(const DedupParams& p, long long v, int lane) {
+  DedupRegs<N> r;
+  dedup_load<N>(r, p, v, lane, false);
+  return dedup128_regs<N, EVEN, false>(p, v, lane, r, nullptr);
 }
 
 }  // namespace sshopm

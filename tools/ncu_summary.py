@@ -5,7 +5,7 @@ from collections import defaultdict
 rep = sys.argv[1]
 def page(*a):
     return subprocess.run(['ncu', '-i', rep] + list(a), capture_output=True, text=True).stdout
-r = list(csv.reader(io.StringIO(page('--page', 'raw', '--csv'))))
+r = list(csv.reader(io.StringIO(page('--page', 'raw', '--csv', '--print-units', 'base'))))
 d = dict(zip(r[0], r[2] if len(r) > 2 else r[1]))
 keys = ['gpu__time_duration.sum', 'sm__throughput.avg.pct_of_peak_sustained_elapsed',
         'smsp__issue_active.avg.pct_of_peak_sustained_active', 'sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active',
