@@ -325,7 +325,7 @@ def main():
                 "x": torch.empty((Nloc, KMAX, n), dtype=torch.float32).pin_memory(),
                 "mult": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory(),
                 "rep": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()}
-        chunk = a.e2e_chunk or min(65536, max(4096, Nloc // 32))
+        chunk = a.e2e_chunk or min(65536, max(4096, Nloc // 16))   # the library default (host_pipeline.cu)
         solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
                         chunk_tensors=chunk, out=outs)
         if world > 1:

@@ -79,7 +79,8 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   const bool raw = h_raw_lambda || h_raw_x || h_raw_iters || h_raw_converged;
   if (raw && !(h_raw_lambda && h_raw_x && h_raw_iters && h_raw_converged)) return SSHOPM_EINVAL;
   const int n = h->n, U = h->U;
-  long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 32;   // default: ~32 chunks, 4K..64K tensors
+  // default: ~16 chunks of 4K..64K tensors (C2 e2e: 16K 6.75 ms, 32K 5.88, 64K 5.65, 128K 6.33; profiles/r1/e2e_sweep.txt)
+  long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 16;
   if (chunk_tensors <= 0) chunk = chunk < 4096 ? 4096 : (chunk > 65536 ? 65536 : chunk);
   if (chunk > N) chunk = N;
 

@@ -97,7 +97,7 @@ cudaError_t apply(long long n_items, const float4* packed, const float* x, float
 
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
-                      Sh::BFORM ? 1 : 0, steps_per_trip<M, N>() == 3 ? 8 : 10, 1,   // refill threshold K (swept on B200)
+                      Sh::BFORM ? 1 : 0, steps_per_trip<M, N>() == 3 ? 8 : 6, 1,   // refill threshold K (swept on B200, profiles/r1/solve_variants.txt)
                       class_index, occupancy, pack, solve, classify, apply};
 }  // namespace
 
