@@ -113,7 +113,11 @@ typedef struct {
   void* d_workspace;               /* optional caller-owned device workspace, 256-byte aligned, >= sshopm_workspace_size */
   size_t workspace_bytes;          /* its size; a too-small or misaligned workspace returns EINVAL */
   int schedule;                    /* 0 default, 1 = item per lane (warps claim chunks of whole tensors),
-                                      2 = tensor per lane (a lane walks one tensor's starts); results identical */
+                                      2 = tensor per lane (a lane walks one tensor's starts); results identical.
+                                      Table-driven general kernel (the only path for (m, n) without a compiled
+                                      kernel): 3 = item per lane (default when its per-lane
+                                      shared-memory arrays fit), 4 = block per tensor, thread per start (the
+                                      paper's mapping); 3 and 4 also force it on compiled shapes. */
   int fuse_dedup;                  /* sshopm_solve_dedup only: 1 = cluster inside the solve kernel (fused),
                                       0 = default (two passes; faster on B200); results identical */
   int alpha_mode;                  /* shift: 0 = the scalar alpha argument (default);

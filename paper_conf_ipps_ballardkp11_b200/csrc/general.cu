@@ -141,11 +141,216 @@ __global__ void __launch_bounds__(128) sshopm_general_apply_kernel(const GenPara
   }
 }
 
+// ------------------------------------------------ item-per-lane general kernel --
+// The default table-driven path (any (m, n) whose per-lane arrays fit in shared
+// memory).  Same stopping rule, shift and outputs as every other kernel, but
+// scheduled like the unrolled solve kernel: persistent warps claim chunks of
+// whole tensors, one lane = one (tensor, start) item, stopped lanes are refilled
+// in batches.  Evaluation is Eq. 6 regrouped by the degree-(m-1) monomial q
+// (DESIGN.md "Evaluation"): (A x^{m-1})_j = sum_q [(m-1)!/q!] a_{class(q+e_j)} x^q,
+// with every monomial of degree 1..m-1 built from its prefix by one multiply
+// (table `recipe`, lexicographic within a degree; degree 1 is x itself).
+// Per-lane arrays live in shared memory, lane-interleaved (element c of lane l at
+// word 32 c + l) so every access is bank-conflict free: the tensor row (U
+// entries) and the monomials (L words, the first n of which hold x).
+struct Gen2Params {
+  const float* entries;      // [N][U]
+  const float* starts;       // [S][n] raw
+  const uint32_t* recipe;    // [L]: (parent | var << 16) for i >= n (degree >= 2)
+  const float* coef;         // [Q]: (m-1)!/q!
+  const uint32_t* cls;       // [Q][n]: byte offset 128 * class(q + e_j) in the lane-interleaved row
+  const int* cls_mult;       // [U]: m!/k! (automatic shift)
+  float* out_lambda;
+  float* out_x;
+  int32_t* out_iters;
+  uint8_t* out_conv;
+  unsigned long long* total_iters;
+  const float* alpha_in;     // alpha_mode 1
+  unsigned int* counter;     // chunk counter (zeroed by the host)
+  long long N, n_chunks;
+  int chunk_tensors;
+  int m, n, U, S, L, Q;
+  float alpha, tol;
+  int alpha_mode, maxit, refill_k;
+};
+
+__device__ __forceinline__ float gen_rsqrt_ftz(float v) {
+  float r;
+  asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(v));
+  return r;
+}
+
+template <int NMAX>
+__global__ void __launch_bounds__(256) sshopm_general2_kernel(const Gen2Params p) {
+  extern __shared__ float gsm[];
+  const int n = p.n, U = p.U, L = p.L, Q = p.Q;
+  const int lane = threadIdx.x & 31;
+  const uint32_t FULL = 0xffffffffu;
+  uint32_t ltmask;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(ltmask));
+  // tables (shared by the CTA), then per-warp lane-interleaved arrays
+  uint32_t* t_rec = reinterpret_cast<uint32_t*>(gsm);
+  float* t_coef = reinterpret_cast<float*>(t_rec + L);
+  uint32_t* t_cls = reinterpret_cast<uint32_t*>(t_coef + Q);
+  int* t_mult = reinterpret_cast<int*>(t_cls + Q * n);
+  for (int i = threadIdx.x; i < L; i += blockDim.x) t_rec[i] = p.recipe[i];
+  for (int i = threadIdx.x; i < Q; i += blockDim.x) t_coef[i] = p.coef[i];
+  for (int i = threadIdx.x; i < Q * n; i += blockDim.x) t_cls[i] = p.cls[i];
+  for (int i = threadIdx.x; i < U; i += blockDim.x) t_mult[i] = p.cls_mult[i];
+  __syncthreads();
+  char* wbase = reinterpret_cast<char*>(t_mult + U) + (size_t)(threadIdx.x >> 5) * 32 * (U + L) * 4 + lane * 4;
+  char* row = wbase;                                   // row[c] at row + 128 c
+  char* mono = wbase + (size_t)U * 128;                // mono[i] at mono + 128 i; mono[0..n) = x
+#define ROW(c) (*reinterpret_cast<float*>(row + (size_t)(c) * 128))
+#define MONO(i) (*reinterpret_cast<float*>(mono + (size_t)(i) * 128))
+
+  // warp-uniform chunk state (global item indices)
+  long long c_next = 0, c_end = 0;
+  bool exhausted = false;
+  uint32_t k_eff = (uint32_t)p.refill_k;
+  float x[NMAX];
+#pragma unroll
+  for (int j = 0; j < NMAX; ++j) x[j] = 0.f;
+  float lam = 0.f, lamp = 0.f, la = 0.f, ls = 1.f;
+  int k = 0;
+  bool has = false, stop = true, conv = false;
+  long long item = 0;
+  uint32_t it_sum = 0;
+  const long long S = p.S;
+  const int offD = L - Q;
+
+  for (;;) {
+    const uint32_t smask = __ballot_sync(FULL, stop);
+    const uint32_t cnt = __popc(smask);
+    if (cnt >= k_eff) {
+      if (stop && has) {
+        p.out_lambda[item] = lam;
+#pragma unroll
+        for (int j = 0; j < NMAX; ++j)
+          if (j < n) p.out_x[item * n + j] = x[j];
+        p.out_iters[item] = k;
+        p.out_conv[item] = conv ? 1 : 0;
+        it_sum += (uint32_t)k;
+      }
+      const long long avail = c_end - c_next;
+      long long n_begin = 0, n_end = 0;
+      if (!exhausted && (long long)cnt > avail) {
+        unsigned int ch = 0;
+        if (lane == 0) ch = atomicAdd(p.counter, 1u);
+        ch = __shfl_sync(FULL, ch, 0);
+        if ((long long)ch < p.n_chunks) {
+          const long long t0 = (long long)ch * p.chunk_tensors;
+          const long long t1 = min(p.N, t0 + p.chunk_tensors);
+          n_begin = t0 * S;
+          n_end = t1 * S;
+        }
+      }
+      const long long rank = __popc(smask & ltmask);
+      const long long t = rank < avail ? c_next + rank : n_begin + (rank - avail);
+      const bool ok = stop && !exhausted && (rank < avail || t < n_end);
+      if (ok) {
+        item = t;
+        const long long v = t / S;
+        const int s = (int)(t - v * S);
+        const float* e = p.entries + v * U;
+        for (int c = 0; c < U; ++c) ROW(c) = __ldg(e + c);
+        float nn = 0.f;
+#pragma unroll
+        for (int j = 0; j < NMAX; ++j)
+          if (j < n) { x[j] = __ldg(p.starts + (size_t)s * n + j); nn = fmaf(x[j], x[j], nn); }
+        const float r0 = nn > 0.f ? rsqrtf(nn) : 0.f;                          // R7
+#pragma unroll
+        for (int j = 0; j < NMAX; ++j)
+          if (j < n) { x[j] *= r0; MONO(j) = x[j]; }
+        float a = p.alpha;
+        if (p.alpha_mode == 1) {
+          a = __ldg(p.alpha_in + v);
+        } else if (p.alpha_mode >= 2) {                                       // R17 bound
+          float b = 0.f;
+          for (int c = 0; c < U; ++c) b = fmaf((float)t_mult[c], fabsf(ROW(c)), b);
+          b *= (float)(p.m - 1);
+          a = p.alpha_mode == 2 ? b : -b;
+        }
+        ls = a >= 0.f ? 1.f : -1.f;                                           // R5
+        la = fabsf(a);
+        k = 0;
+        lamp = __int_as_float(0x7fffffff);                                    // NaN: first test never fires
+      }
+      has = stop ? ok : has;
+      if (!exhausted) {
+        if ((long long)cnt > avail) {
+          if (n_end == 0) { exhausted = true; k_eff = 32u; }
+          c_next = min(n_begin + ((long long)cnt - avail), n_end);
+          c_end = n_end;
+        } else {
+          c_next += cnt;
+        }
+      }
+      if (exhausted && __ballot_sync(FULL, has) == 0u) break;
+    }
+
+    // ---- one SS-HOPM step (Fig. 1) ----
+#pragma unroll 4
+    for (int i = n; i < L; ++i) {                                             // monomials of degree 2..m-1
+      const uint32_t r = t_rec[i];
+      MONO(i) = MONO(r & 0xffffu) * MONO(r >> 16);
+    }
+    float g[NMAX];
+#pragma unroll
+    for (int j = 0; j < NMAX; ++j) g[j] = 0.f;
+    for (int q = 0; q < Q; ++q) {                                             // Eq. 6 by monomial
+      const float cm = t_coef[q] * MONO(offD + q);
+      const uint32_t* cq = t_cls + q * n;
+#pragma unroll
+      for (int j = 0; j < NMAX; ++j)
+        if (j < n) g[j] = fmaf(*reinterpret_cast<const float*>(row + cq[j]), cm, g[j]);
+    }
+    lam = 0.f;
+#pragma unroll
+    for (int j = 0; j < NMAX; ++j)
+      if (j < n) lam = fmaf(x[j], g[j], lam);                                // lambda_k = x_k . g
+    conv = fabsf(lam - lamp) <= p.tol * fmaxf(1.0f, fabsf(lam));              // R2
+    float nn = 0.f;
+#pragma unroll
+    for (int j = 0; j < NMAX; ++j)
+      if (j < n) { g[j] = fmaf(la, x[j], ls * g[j]); nn = fmaf(g[j], g[j], nn); }   // xhat = +-(g + alpha x)
+    const bool deg = !(nn >= 1.17549435e-38f);                               // R6
+    stop = (!has) | conv | (k >= p.maxit) | deg;
+    const float r = gen_rsqrt_ftz(nn);
+    if (!stop) {
+#pragma unroll
+      for (int j = 0; j < NMAX; ++j)
+        if (j < n) { x[j] = g[j] * r; MONO(j) = x[j]; }
+      lamp = lam;
+      ++k;
+    }
+  }
+#undef ROW
+#undef MONO
+  if (p.total_iters) {
+    unsigned long long ws = it_sum;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(FULL, ws, o);
+    if (lane == 0) atomicAdd(p.total_iters, ws);
+  }
+}
+
 // ------------------------------------------------------------------ host --
 static long long binom_ll(int a, int b) {
   if (b < 0 || b > a) return 0;
   long long r = 1;
   for (int i = 1; i <= b; ++i) r = r * (a - b + i) / i;
+  return r;
+}
+
+// lexicographic rank of a nondecreasing length-d tuple over {0..n-1} among all such tuples
+static long long lex_rank(const int* I, int d, int n) {
+  long long r = 0;
+  int lo = 0;
+  for (int p = 0; p < d; ++p) {
+    for (int v = lo; v < I[p]; ++v) r += binom_ll((d - p - 1) + (n - v) - 1, d - p - 1);
+    lo = I[p];
+  }
   return r;
 }
 
@@ -180,6 +385,55 @@ GeneralTables* general_create(int m, int n) {
     for (int k = j + 1; k < m; ++k) I[k] = I[j];
   }
   const long long Q = binom_ll(m + n - 2, m - 1);
+  // item-per-lane kernel: monomials of degree 1..m-1 (lexicographic within a degree) built from
+  // their prefix, and for each degree-(m-1) monomial q its coefficient (m-1)!/q! and the classes
+  // of q + e_j (P:L180 for sigma)
+  const int D = m - 1;
+  const long long L = binom_ll(D + n, D) - 1;
+  if (L + U <= kGen2MaxWords) {
+    t->L = (int)L;
+    t->Q = (int)Q;
+    t->recipe = new (std::nothrow) uint32_t[L];
+    t->coef = new (std::nothrow) float[Q];
+    t->cls = new (std::nothrow) uint32_t[Q * n];
+    if (!t->recipe || !t->coef || !t->cls) { general_destroy(t); return nullptr; }
+    long long off = 0, prev_off = 0;
+    for (int d = 1; d <= D; ++d) {
+      int T[kGenMaxM] = {};
+      const long long cnt = binom_ll(d + n - 1, d);
+      for (long long i = 0; i < cnt; ++i) {
+        if (d == 1) t->recipe[off + i] = 0;
+        else t->recipe[off + i] = (uint32_t)(prev_off + lex_rank(T, d - 1, n)) | ((uint32_t)T[d - 1] << 16);
+        if (d == D) {
+          const long long q = i;
+          long long den = 1;
+          int run = 1;
+          for (int k = 1; k < d; ++k) { if (T[k] == T[k - 1]) { ++run; den *= run; } else run = 1; }
+          long long fd = 1;
+          for (int k = 2; k <= D; ++k) fd *= k;
+          t->coef[q] = (float)((double)fd / (double)den);
+          for (int j = 0; j < n; ++j) {                    // class of q + e_j: insert j into the sorted tuple
+            int C[kGenMaxM + 1];
+            int w = 0;
+            bool put = false;
+            for (int k = 0; k < d; ++k) {
+              if (!put && j <= T[k]) { C[w++] = j; put = true; }
+              C[w++] = T[k];
+            }
+            if (!put) C[w++] = j;
+            t->cls[q * n + j] = (uint32_t)(128 * lex_rank(C, m, n));
+          }
+        }
+        int k2 = d - 1;                                     // Fig. 4 successor
+        while (k2 >= 0 && T[k2] == n - 1) --k2;
+        if (k2 < 0) break;
+        T[k2] += 1;
+        for (int r = k2 + 1; r < d; ++r) T[r] = T[k2];
+      }
+      prev_off = off;
+      off += cnt;
+    }
+  }
   t->paper_flops = (long long)(m + 2) * U + (long long)(m + 1) * n * Q + 5LL * n;
   // executed per update: per class ~ (m suffix + m prefix + 3 per unique index) + lambda/shift/normalise
   t->exec_flops = U * (2LL * m + 3LL * n / 2) + 7LL * n;
@@ -190,6 +444,9 @@ void general_destroy(GeneralTables* t) {
   if (!t) return;
   delete[] t->idx;
   delete[] t->mult;
+  delete[] t->recipe;
+  delete[] t->coef;
+  delete[] t->cls;
   delete t;
 }
 
@@ -210,9 +467,87 @@ int general_upload(const GeneralTables* t, void* dev, cudaStream_t st, const uin
   return SSHOPM_OK;
 }
 
+template <int NMAX>
+static cudaError_t launch_general2(const Gen2Params& p, int warps, int smem, cudaStream_t st) {
+  cudaError_t e = cudaFuncSetAttribute(sshopm_general2_kernel<NMAX>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  int bps = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, sshopm_general2_kernel<NMAX>, 32 * warps, smem);
+  if (e != cudaSuccess) return e;
+  if (bps < 1) return cudaErrorInvalidConfiguration;
+  long long grid = (long long)device_sms() * bps;
+  const long long need = (p.n_chunks + 3) / 4;            // >= 4 chunks per warp-group on average
+  if (grid > need) grid = need > 0 ? need : 1;
+  sshopm_general2_kernel<NMAX><<<(int)grid, 32 * warps, smem, st>>>(p);
+  return cudaGetLastError();
+}
+
+// item-per-lane general kernel (tables in the handle's host copy, uploaded per call)
+static int general2_solve(const GeneralTables* t, int64_t N, const float* d_entries, int S, const float* d_starts,
+                          float alpha, float tol, int maxit, float* d_lambda, float* d_x, int32_t* d_iters,
+                          uint8_t* d_conv, const sshopm_solve_opts* opts, cudaStream_t st, int warps, int smem) {
+  const int alpha_mode = opts ? opts->alpha_mode : 0;
+  if (alpha_mode < 0 || alpha_mode > 3 || (alpha_mode == 1 && !opts->d_alpha)) return SSHOPM_EINVAL;
+  const size_t b_rec = ((size_t)t->L * 4 + 255) / 256 * 256, b_coef = ((size_t)t->Q * 4 + 255) / 256 * 256;
+  const size_t b_cls = ((size_t)t->Q * t->n * 4 + 255) / 256 * 256, b_mult = ((size_t)t->U * 4 + 255) / 256 * 256;
+  char* tab = nullptr;
+  cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&tab), 256 + b_rec + b_coef + b_cls + b_mult, st);
+  if (e != cudaSuccess) return e == cudaErrorMemoryAllocation ? SSHOPM_ENOMEM : cuda_fail(e, "general: malloc");
+  Gen2Params p;
+  memset(&p, 0, sizeof(p));
+  p.counter = reinterpret_cast<unsigned int*>(tab);
+  p.recipe = reinterpret_cast<const uint32_t*>(tab + 256);
+  p.coef = reinterpret_cast<const float*>(tab + 256 + b_rec);
+  p.cls = reinterpret_cast<const uint32_t*>(tab + 256 + b_rec + b_coef);
+  p.cls_mult = reinterpret_cast<const int*>(tab + 256 + b_rec + b_coef + b_cls);
+  e = cudaMemsetAsync(tab, 0, 256, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.recipe, t->recipe, (size_t)t->L * 4, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.coef, t->coef, (size_t)t->Q * 4, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.cls, t->cls, (size_t)t->Q * t->n * 4, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.cls_mult, t->mult, (size_t)t->U * 4, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) { cudaFreeAsync(tab, st); return cuda_fail(e, "general: table upload"); }
+  p.entries = d_entries;
+  p.starts = d_starts;
+  p.out_lambda = d_lambda;
+  p.out_x = d_x;
+  p.out_iters = d_iters;
+  p.out_conv = d_conv;
+  p.total_iters = opts ? opts->d_total_iters : nullptr;
+  p.alpha_in = alpha_mode == 1 ? opts->d_alpha : nullptr;
+  p.N = N;
+  p.chunk_tensors = chunk_tensors_for(S);
+  p.n_chunks = (N + p.chunk_tensors - 1) / p.chunk_tensors;
+  p.m = t->m;
+  p.n = t->n;
+  p.U = t->U;
+  p.S = S;
+  p.L = t->L;
+  p.Q = t->Q;
+  p.alpha = alpha;
+  p.tol = tol;
+  p.alpha_mode = alpha_mode;
+  p.maxit = maxit;
+  const int k = (opts && opts->refill_threshold > 0) ? opts->refill_threshold : 4;
+  p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
+  e = t->n <= 4 ? launch_general2<4>(p, warps, smem, st)
+    : t->n <= 8 ? launch_general2<8>(p, warps, smem, st) : launch_general2<16>(p, warps, smem, st);
+  cudaFreeAsync(tab, st);
+  if (e != cudaSuccess) return cuda_fail(e, "general: launch");
+  return SSHOPM_OK;
+}
+
 int general_solve(const GeneralTables* t, int64_t N, const float* d_entries, int S, const float* d_starts, float alpha,
                   float tol, int maxit, float* d_lambda, float* d_x, int32_t* d_iters, uint8_t* d_conv,
                   const sshopm_solve_opts* opts, cudaStream_t st) {
+  if (t->recipe && !(opts && opts->schedule == 4)) {           // item-per-lane kernel unless forced off
+    const int tables = (t->L + t->Q + t->Q * t->n + t->U) * 4;
+    const int per_warp = 32 * (t->U + t->L) * 4;
+    int warps = (200 * 1024 - tables) / per_warp;
+    if (warps > 8) warps = 8;
+    if (warps >= 1)
+      return general2_solve(t, N, d_entries, S, d_starts, alpha, tol, maxit, d_lambda, d_x, d_iters, d_conv, opts, st,
+                            warps, tables + warps * per_warp);
+  }
   const int block = 128;
   const int smem = general_smem(t, block, true);
   if (smem > 200 * 1024) return SSHOPM_EUNSUPPORTED;

@@ -10,11 +10,18 @@ constexpr int kGenMaxM = 16;     // order limit of the general kernel
 constexpr int kGenMaxN = 16;     // dimension limit
 constexpr long long kGenMaxU = 1 << 16;
 
+constexpr long long kGen2MaxWords = 1500;   // item-per-lane kernel: per-lane shared words U + L (32 lanes per warp)
+
 struct GeneralTables {           // host copies; uploaded per call (handles own no device memory)
   int m = 0, n = 0, U = 0;
   uint8_t* idx = nullptr;        // [U][m] index representations, lexicographic (Fig. 4 walk)
   int* mult = nullptr;           // [U] m!/k! (Property 2)
   long long paper_flops = 0, exec_flops = 0;
+  // item-per-lane kernel (null when U + L > kGen2MaxWords: the block-per-tensor kernel is used)
+  int L = 0, Q = 0;              // monomials of degree 1..m-1; those of degree m-1
+  uint32_t* recipe = nullptr;    // [L] parent | var << 16 (degree >= 2)
+  float* coef = nullptr;         // [Q] (m-1)!/q!
+  uint32_t* cls = nullptr;       // [Q][n] 128 * class(q + e_j)
 };
 
 GeneralTables* general_create(int m, int n);

@@ -235,7 +235,8 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const Launchers* L = h->L;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
-  if (!L || (opts && opts->schedule == 3)) {                     // table-driven general kernel (any (m, n))
+  if (opts && (opts->schedule < 0 || opts->schedule > 4)) return SSHOPM_EINVAL;
+  if (!L || (opts && opts->schedule >= 3)) {                     // table-driven general kernel (any (m, n))
     if (!h->gen) return SSHOPM_EUNSUPPORTED;
     int rc = general_solve(h->gen, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
                            d_out_converged, opts, st);
@@ -260,7 +261,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const bool wide = (long long)N * S >= (1LL << 31) - (1LL << 20);
   // schedule: 1 = item per lane (chunks of whole tensors), 2 = tensor per lane
   int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
-  if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;   // 3 (general) handled above
+  if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;   // 3 / 4 (general) handled above
   if (shift == 3) schedule = 1;                                  // per-tensor alpha: schedule 1 only
   int bps = 0;
   cudaError_t e = cached_occupancy(h, shift, wide, schedule, &bps);

@@ -366,27 +366,34 @@ def test_general_apply_exact(dev, m, n):
     assert np.array_equal(lam.cpu().numpy().astype(np.float64), lam_ref)
 
 
-@pytest.mark.parametrize("m,n,V,alpha", [(5, 4, 24, 4.0), (6, 4, 16, 0.5), (3, 6, 16, 3.0), (10, 2, 32, 0.5), (4, 8, 8, 0.0)])
-def test_general_solve_parity(dev, m, n, V, alpha):
+@pytest.mark.parametrize("m,n,V,alpha", [(5, 4, 24, 4.0), (6, 4, 16, 0.5), (3, 6, 16, 3.0), (10, 2, 32, 0.5), (4, 8, 8, 0.0),
+                                         (6, 5, 6, 0.5), (3, 9, 8, 1.0)])
+@pytest.mark.parametrize("schedule", [0, 4])
+def test_general_solve_parity(dev, m, n, V, alpha, schedule):
+    """(m, n) without a compiled kernel: item-per-lane general kernel (default; n = 9 takes its
+    16-wide register variant) and the block-per-tensor one (schedule 4) vs the oracle."""
     ent = syn.gen_voxels(m, n, 0, V, 3) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 3)
     st = syn.gen_starts(64, n, 1)
-    gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 200)
+    gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 200, schedule=schedule)
     _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 200, gpu), 0.05)
 
 
-def test_general_kernel_on_compiled_shape(dev):
-    """opts.schedule = 3 forces the table-driven kernel on (4,3): same contract vs the oracle."""
-    m, n = 4, 3
-    ent = syn.gen_voxels(m, n, 0, 256, 0)
-    st = syn.gen_starts(128, n, 0)
-    gpu = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, schedule=3)
-    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, gpu))
-    # automatic shift: the general and unrolled kernels agree (different FP32 summation orders)
-    a3 = _solve(dev, m, n, ent[:32], st, "auto_max", 1e-6, 300, schedule=3)
-    a1 = _solve(dev, m, n, ent[:32], st, "auto_max", 1e-6, 300, schedule=1)
-    both = (a3[3] == 1) & (a1[3] == 1)
-    assert both.mean() > 0.5
-    assert np.all(np.abs(a3[0][both] - a1[0][both]) <= 1e-4 * np.maximum(1, np.abs(a1[0][both])))
+@pytest.mark.parametrize("shift", ["auto_max", "auto_min"])
+def test_general_item_kernel_shift_modes(dev, shift):
+    """Item-per-lane general kernel with the automatic convex / concave shifts and ragged chunks
+    (S = 100, V = 37): in fixed-K mode (tol < 0, 50 updates) its lambda_K equals the
+    block-per-tensor kernel's up to FP32 summation order (both compute the same shift, R17,
+    in the same class order); scalar shifts are covered against the oracle above."""
+    m, n, V, S = 5, 4, 37, 100
+    ent = syn.gen_uniform_tensors(m, n, V, 11)
+    st = syn.gen_starts(S, n, 2)
+    a = _solve(dev, m, n, ent, st, shift, -1.0, 50, schedule=3)
+    b = _solve(dev, m, n, ent, st, shift, -1.0, 50, schedule=4)
+    assert np.all(a[2] == 50) and np.all(b[2] == 50) and not a[3].any()
+    assert np.all(np.abs(a[0] - b[0]) <= 1e-4 * np.maximum(1, np.abs(b[0])))
+    if shift == "auto_max":   # convex shift: lambda_k nondecreasing, so lambda_K >= lambda_0 = A x0^m
+        lam0 = _solve(dev, m, n, ent, st, shift, -1.0, 0, schedule=3)[0]
+        assert np.all(a[0] >= lam0 - 1e-4 * np.maximum(1, np.abs(lam0)))
 
 
 # ------------------------------------------------------------ classification --
