@@ -54,6 +54,10 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-voxels", type=int, default=0)
     ap.add_argument("--e2e-chunk", type=int, default=0, help="tensors per run_host chunk (0: auto)")
+    ap.add_argument("--gather-chunks", type=int, default=0,
+                    help="N > 1: solve+dedup the rank's range in C chunks and gather chunk i on a side stream "
+                         "while chunk i+1 solves (0: 4 when N > 1, else 1)")
+    ap.add_argument("--dump-records", default="", help="rank 0: save the gathered dedup records (.npz) after the run")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process group backend for N > 1 (gloo: exercise the multi-rank path on one GPU)")
     return ap.parse_args()
@@ -236,40 +240,64 @@ def main():
     xo = torch.empty((Nloc, S, n), dtype=torch.float32, device=dev)
     it = torch.empty((Nloc, S), dtype=torch.int32, device=dev)
     cv = torch.empty((Nloc, S), dtype=torch.uint8, device=dev)
-    # dedup records packed in one int32 buffer so a single collective moves them (sharding.py)
-    rec = torch.empty(SH.record_words(Nloc, KMAX, n), dtype=torch.int32, device=dev)
-    views = SH.record_views(rec, Nloc, KMAX, n)
+    # dedup records: one int32 block per chunk so one collective moves a chunk (sharding.py); with
+    # N > 1 chunk c's gather runs on a side stream while chunk c+1 solves (SURVEY.md 8(e) overlap)
+    n_chunks = a.gather_chunks or (4 if world > 1 else 1)
+    bounds = SH.chunk_bounds(Nloc, n_chunks)
+    n_chunks = len(bounds)
+    rec = torch.empty(SH.chunked_record_words(Nloc, n_chunks, KMAX, n)[0], dtype=torch.int32, device=dev)
+    blocks = SH.chunked_record_views(rec, Nloc, n_chunks, KMAX, n)
     titers = torch.zeros(1, dtype=torch.int64, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
+    side = torch.cuda.Stream(device=dev)
+    done = [torch.cuda.Event() for _ in range(n_chunks)]
+    gathered = [None] * n_chunks
 
-    def run_path(count_iters=False, mid_event=None):
-        """One pass of the hot path: solve (A0-A7) + dedup (A8).  mid_event is recorded between the
-        solve and the dedup launches (two-pass forms) so the solve kernel is timed on its own."""
+    def run_chunk(c, count_iters=False, ev=None):
+        """One pass of the hot path over chunk c: solve (A0-A7) + dedup (A8).  ev = (start, mid) events
+        recorded around the solve launches (two-pass forms) so the solve kernel is timed on its own."""
         ti = titers if count_iters else None
+        v0, v1 = bounds[c]
+        views = blocks[c][1]
+        o = (lam[v0:v1], xo[v0:v1], it[v0:v1], cv[v0:v1])
+        if ev is not None:
+            ev[0].record(stream)
         if a.unfused:
-            solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=(lam, xo, it, cv),
+            solver.solve(ent[v0:v1], st, cfg["alpha"], cfg["tol"], cfg["maxit"], out=o,
                          refill_threshold=a.refill, total_iters=ti, schedule=a.schedule)
-            if mid_event is not None:
-                mid_event.record(stream)
-            solver.dedup(lam, xo, cv, LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
+            if ev is not None:
+                ev[1].record(stream)
+            solver.dedup(*o[:2], o[3], LAM_TOL, ANG_TOL, KMAX, out=tuple(views))
         else:
-            solver.solve_dedup(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
-                               out=(lam, xo, it, cv), dedup_out=tuple(views), refill_threshold=a.refill,
+            solver.solve_dedup(ent[v0:v1], st, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
+                               out=o, dedup_out=tuple(views), refill_threshold=a.refill,
                                total_iters=ti, schedule=a.schedule, fused=a.fused)
+            if ev is not None:
+                ev[1].record(stream)
+        if world > 1:
+            gather(c)
+
+    def gather(c):
+        block = blocks[c][0]
+        if a.backend == "nccl":                           # A9: NCCL gather of chunk c on the side stream
+            done[c].record(stream)
+            with torch.cuda.stream(side):
+                side.wait_event(done[c])
+                gathered[c] = SH.gather_records(block, rank, world)
+        else:                                             # gloo: stage through host memory (no overlap)
+            gathered[c] = SH.gather_records(block.cpu(), rank, world)
+
+    def run_path(count_iters=False, evs=None):
+        for c in range(n_chunks):
+            run_chunk(c, count_iters, None if evs is None else evs[c])
+        if world > 1:
+            stream.wait_stream(side)                      # the step ends when the last gather has landed
 
     def step(count_iters=False):
         if count_iters:
             titers.zero_()
         run_path(count_iters)
-        if world > 1:
-            gather()
-
-    def gather():
-        if a.backend == "nccl":
-            SH.gather_records(rec, rank, world)
-        else:                                             # gloo: stage through host memory
-            SH.gather_records(rec.cpu(), rank, world)
 
     for _ in range(max(a.warmup, 3)):
         step()
@@ -277,8 +305,10 @@ def main():
     torch.cuda.synchronize()
     iters_local = int(titers.item())
 
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
-           torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    def tev():
+        return torch.cuda.Event(enable_timing=True)
+    ev = [(tev(), tev()) for _ in range(a.steps)]
+    cev = [[(tev(), tev()) for _ in range(n_chunks)] for _ in range(a.steps)]   # per-chunk solve windows
     l0 = solver.launch_count()
     if world > 1:
         dist.barrier()
@@ -288,21 +318,18 @@ def main():
             if i % 4 == 2:
                 clk.sample_now()                          # host-side NVML query: outside the event window
             flush.zero_()
-            e0, e1, e2 = ev[i]
+            e0, e2 = ev[i]
             e0.record(stream)
-            run_path(mid_event=e1)
-            if not a.unfused:
-                e1.record(stream)
-            if world > 1:
-                gather()
+            run_path(evs=cev[i])
             e2.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     launches = solver.launch_count() - l0
-    t_step = [e0.elapsed_time(e2) for e0, e1, e2 in ev]
-    t_solve = [e0.elapsed_time(e1) for e0, e1, e2 in ev]   # pack + solve kernels (with --solve-dedup: the whole call)
+    t_step = [e0.elapsed_time(e2) for e0, e2 in ev]
+    # pack + solve kernels of every chunk (with --solve-dedup: the whole call)
+    t_solve = [sum(s0.elapsed_time(s1) for s0, s1 in cs) for cs in cev]
     tot_ms = float(sum(t_step))
     cdev = dev if a.backend == "nccl" else torch.device("cpu")
     stats = torch.tensor([tot_ms, float(iters_local), float(sum(t_solve))], dtype=torch.float64, device=cdev)
@@ -314,6 +341,13 @@ def main():
         tot_ms, solve_ms, iters_all = float(tmax[0]), float(tmax[1]), float(itsum[0])
     else:
         solve_ms, iters_all = float(stats[2]), float(stats[1])
+
+    if a.dump_records and rank == 0:
+        if world > 1:
+            merged = SH.merge_chunked(gathered, Nloc, n_chunks, KMAX, n)
+        else:
+            merged = SH.merge_chunked([[blk] for blk, _ in blocks], Nloc, n_chunks, KMAX, n)
+        np.savez(a.dump_records, **dict(zip(("count", "lam", "x", "mult", "rep"), merged)))
 
     # end to end through the C ABI on host buffers (pinned), per step
     e2e = None
@@ -360,7 +394,13 @@ def main():
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
     fmax = pk.get("sm_max_mhz") or clk.max_mhz or 1965.0
     peak_tflops = sms * 128 * 2 * fmax * 1e6 / 1e12
-    achieved = Fx * iters_local * a.steps / (solve_ms / 1e3) / 1e12     # rank-local solve kernel
+    # algorithmic flops of one solve: every (tensor, start) lane evaluates lambda_0 = x_0 . A x_0^{m-1}
+    # (reading R1) and then, per update k = 1..iters, one normalisation (+ shift) and one evaluation:
+    # Fx per update + Fe for lambda_0; paper-style `value` keeps lambda_0 excluded (R12)
+    Fu = (2 * n - 1) + n + (2 * n if cfg["alpha"] != 0 else 0)          # ||xhat||^2, scale, shift
+    Fe = Fx - Fu                                                          # monomials + 2*T1 + lambda
+    alg_flops = Fx * iters_local + Fe * Nloc * S
+    achieved = alg_flops * a.steps / (solve_ms / 1e3) / 1e12             # rank-local solve kernel
     traffic = fma_pct = None
     tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tf):
@@ -386,7 +426,8 @@ def main():
                    "flop_count": "paper-style F_paper(m,n) x sum(iters), reading R12",
                    "l2": "flushed between timed steps (512 MiB write outside the events)",
                    "parallelism": f"tensor-range shards x{world}" +
-                                  (f" + {a.backend.upper()} gather of dedup records" if world > 1 else "")},
+                                  (f" + {a.backend.upper()} gather of dedup records in {n_chunks} chunks "
+                                   f"(chunk i gathered while chunk i+1 solves)" if world > 1 else "")},
         "voxel_solves_per_s": vps,
         "start_solves_per_s": vps * S,
         "mean_iters": iters_all / (Nloc * world * S),
@@ -395,9 +436,11 @@ def main():
                      "frac": achieved / peak_tflops, "traffic": traffic,
                      "kernel": f"sshopm_solve_kernel<{m},{n}>",
                      "peak_basis": f"{sms} SM x 128 FP32 lanes x 2 x {fmax:.0f} MHz (sm_max_mhz)",
-                     "flops_per_update": Fx,
+                     "flops_per_update": Fx, "flops_lambda0_eval": Fe,
+                     "flops_per_launch": alg_flops,
                      "fma_pipe_active_pct_ncu": fma_pct,
-                     "flops_note": "algorithmic FP32 flops per (tensor,start,update): monomials + 2*T1 + lambda + shift + norm + scale (DESIGN.md 7)"},
+                     "flops_note": "algorithmic FP32 flops per launch = flops_per_update x sum(iters) + flops_lambda0_eval x N*S "
+                                   "(update: monomials + 2*T1 + lambda + shift + norm + scale; lambda_0: monomials + 2*T1 + lambda; DESIGN.md 7)"},
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,

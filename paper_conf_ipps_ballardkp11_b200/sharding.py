@@ -6,6 +6,12 @@ solves and dedups it locally, and one collective moves the fixed-size
 per-tensor dedup records to rank 0.  No data-path
 collective exists during the solve.
 
+Overlap: a rank may split its range into C contiguous chunks
+(`chunk_bounds`) with one record block per chunk (`chunked_record_views`);
+chunk i's block is gathered on a side stream while chunk i+1 solves, so only
+the last chunk's gather is exposed.  `merge_chunked` reassembles rank 0's
+gathered blocks in global tensor order.
+
 Record layout (one int32 buffer per rank, so a single collective moves it):
     count [N] i32 | lambda [N, K] f32 | x [N, K, n] f32 | mult [N, K] i32 | rep [N, K] i32
 Float fields are stored bit-for-bit (reinterpreted as int32).  All ranks use
@@ -62,3 +68,51 @@ def merge_records(bufs, n_per_rank, kmax, n, n_total=None):
     if n_total is not None:
         merged = tuple(m[:n_total] for m in merged)
     return merged
+
+
+def chunk_bounds(n_tensors, n_chunks):
+    """[(v0, v1)] of `n_chunks` contiguous, balanced sub-ranges covering [0, n_tensors) (empty ones dropped)."""
+    n_chunks = max(1, min(int(n_chunks), max(1, int(n_tensors))))
+    out = []
+    for c in range(n_chunks):
+        f, k = shard_range(n_tensors, c, n_chunks)
+        if k > 0:
+            out.append((f, f + k))
+    return out
+
+
+def chunked_record_words(n_tensors, n_chunks, kmax, n):
+    """Words of a buffer holding one record block per chunk, each sized for the largest chunk
+    (identical on every rank because all ranks hold the same number of tensors)."""
+    bounds = chunk_bounds(n_tensors, n_chunks)
+    per = max((v1 - v0 for v0, v1 in bounds), default=0)
+    return len(bounds) * record_words(per, kmax, n), per
+
+
+def chunked_record_views(buf, n_tensors, n_chunks, kmax, n):
+    """[(block, views)] per chunk: `block` is the chunk's flat slice of `buf` (what one gather moves),
+    `views` its (count, lambda, x, mult, rep) fields sized for the chunk's own tensor count."""
+    bounds = chunk_bounds(n_tensors, n_chunks)
+    _, per = chunked_record_words(n_tensors, n_chunks, kmax, n)
+    w = record_words(per, kmax, n)
+    out = []
+    for i, (v0, v1) in enumerate(bounds):
+        block = buf[i * w:(i + 1) * w]
+        views = tuple(v[:v1 - v0] for v in record_views(block, per, kmax, n))
+        out.append((block, views))
+    return out
+
+
+def merge_chunked(gathered, n_per_rank, n_chunks, kmax, n):
+    """Rank-0 side: gathered[c][r] = rank r's block of chunk c (from one gather per chunk).
+    Returns global (count, lambda, x, mult, rep) host arrays in tensor order (rank-major, then chunk)."""
+    bounds = chunk_bounds(n_per_rank, n_chunks)
+    _, per = chunked_record_words(n_per_rank, n_chunks, kmax, n)
+    world = len(gathered[0])
+    parts = []
+    for r in range(world):
+        for c, (v0, v1) in enumerate(bounds):
+            b = gathered[c][r]
+            b = b.cpu().numpy() if hasattr(b, "cpu") else np.asarray(b)
+            parts.append(tuple(v[:v1 - v0] for v in record_views(b, per, kmax, n)))
+    return tuple(np.concatenate([p[i] for p in parts], axis=0) for i in range(5))

@@ -35,3 +35,38 @@ def test_bench_two_ranks_gloo():
     assert d["n_gpus"] == 2 and d["scaling"] == "weak"
     assert d["config"]["tensors_total"] == 2 * 65536
     assert d["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
+
+
+def test_chunked_gather_bitwise_equal_to_one_process(tmp_path):
+    """C5 invariant: dedup records gathered from P = 2 ranks, each solving its range in
+    3 chunks, equal bit for bit those of one process solving the whole volume in one call."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import numpy as np
+    import paper_conf_ipps_ballardkp11_b200 as sh
+    import synthetic as syn
+    nloc, kmax = 8192, 4
+    dump = str(tmp_path / "rec.npz")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "1", "--warmup", "3", "--backend", "gloo", "--no-cpu", "--no-e2e",
+           "--voxels", str(nloc), "--gather-chunks", "3", "--dump-records", dump]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    got = np.load(dump)
+    cfg = syn.CONFIGS["C2"]
+    m, n, S = cfg["m"], cfg["n"], cfg["S"]
+    dev = torch.device("cuda:0")
+    ent = torch.from_numpy(syn.gen_voxels(m, n, 0, 2 * nloc, seed=0)).to(dev)
+    st = torch.from_numpy(syn.gen_starts(S, n, seed=0)).to(dev)
+    solver = sh.Solver(m, n)
+    lam, x, it, cv = solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"])
+    ref = solver.dedup(lam, x, cv, 1e-2, 0.05, kmax)
+    torch.cuda.synchronize()
+    for name, a in zip(("count", "lam", "x", "mult", "rep"), ref):
+        a = a.cpu().numpy()
+        b = got[name]
+        assert a.shape == b.shape, name
+        assert np.array_equal(a.view(np.int32) if a.dtype == np.float32 else a,
+                              b.view(np.int32) if b.dtype == np.float32 else b), name
