@@ -115,9 +115,13 @@ typedef struct {
   int schedule;                    /* 0 default, 1 = item per lane (warps claim chunks of whole tensors),
                                       2 = tensor per lane (a lane walks one tensor's starts); results identical.
                                       Table-driven general kernel (the only path for (m, n) without a compiled
-                                      kernel): 3 = item per lane (default when its per-lane
-                                      shared-memory arrays fit), 4 = block per tensor, thread per start (the
-                                      paper's mapping); 3 and 4 also force it on compiled shapes. */
+                                      kernel): 5 = blocked (default): warp per tensor, the
+                                      tensor's coefficient-folded rows once per warp in shared memory, blocks of
+                                      Eq. 6 per degree-(m-2) prefix ("blocked approach"); 3 = item per
+                                      lane, the tensor row per lane in shared memory; 4 = block per tensor,
+                                      thread per start (the paper's mapping); 3-5 also force the
+                                      table-driven path on compiled shapes (5 returns EUNSUPPORTED if its
+                                      shared memory does not fit; the default then falls back to 3, then 4). */
   int fuse_dedup;                  /* sshopm_solve_dedup only: 1 = cluster inside the solve kernel (fused),
                                       0 = default (two passes; faster on B200); results identical */
   int alpha_mode;                  /* shift: 0 = the scalar alpha argument (default);

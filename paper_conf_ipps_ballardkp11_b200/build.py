@@ -52,7 +52,7 @@ def _units():
     for m, n in shapes():
         u.append((os.path.join(CSRC, "sshopm_instance.cu"), os.path.join(BUILD, f"inst_{m}_{n}.o"),
                   [f"-DSSHOPM_M={m}", f"-DSSHOPM_N={n}"]))
-    for src in ("sshopm_api.cu", "host_pipeline.cu", "general.cu"):
+    for src in ("sshopm_api.cu", "host_pipeline.cu", "general.cu", "blocked.cu"):
         u.append((os.path.join(CSRC, src), os.path.join(BUILD, src.replace(".cu", ".o")), []))
     return u
 

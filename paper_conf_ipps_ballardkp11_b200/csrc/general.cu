@@ -390,18 +390,24 @@ GeneralTables* general_create(int m, int n) {
   // of q + e_j (P:L180 for sigma)
   const int D = m - 1;
   const long long L = binom_ll(D + n, D) - 1;
-  if (L + U <= kGen2MaxWords) {
+  if (Q * n <= kBlkMaxT1 && L < 65536) {
     t->L = (int)L;
     t->Q = (int)Q;
+    t->gen2 = (L + U <= kGen2MaxWords);
+    t->P = m >= 3 ? (int)binom_ll(m - 2 + n - 1, m - 2) : 1;
     t->recipe = new (std::nothrow) uint32_t[L];
     t->coef = new (std::nothrow) float[Q];
     t->cls = new (std::nothrow) uint32_t[Q * n];
-    if (!t->recipe || !t->coef || !t->cls) { general_destroy(t); return nullptr; }
+    t->cls_idx = new (std::nothrow) uint32_t[Q * n];
+    t->plast = new (std::nothrow) uint32_t[t->P];
+    if (!t->recipe || !t->coef || !t->cls || !t->cls_idx || !t->plast) { general_destroy(t); return nullptr; }
+    t->plast[0] = 0;                                     // m = 2: the empty prefix (x^0 = 1)
     long long off = 0, prev_off = 0;
     for (int d = 1; d <= D; ++d) {
       int T[kGenMaxM] = {};
       const long long cnt = binom_ll(d + n - 1, d);
       for (long long i = 0; i < cnt; ++i) {
+        if (d == m - 2) t->plast[i] = (uint32_t)T[d - 1];  // blocked kernel: last index of each prefix
         if (d == 1) t->recipe[off + i] = 0;
         else t->recipe[off + i] = (uint32_t)(prev_off + lex_rank(T, d - 1, n)) | ((uint32_t)T[d - 1] << 16);
         if (d == D) {
@@ -421,7 +427,8 @@ GeneralTables* general_create(int m, int n) {
               C[w++] = T[k];
             }
             if (!put) C[w++] = j;
-            t->cls[q * n + j] = (uint32_t)(128 * lex_rank(C, m, n));
+            t->cls_idx[q * n + j] = (uint32_t)lex_rank(C, m, n);
+            t->cls[q * n + j] = 128u * t->cls_idx[q * n + j];
           }
         }
         int k2 = d - 1;                                     // Fig. 4 successor
@@ -433,6 +440,42 @@ GeneralTables* general_create(int m, int n) {
       prev_off = off;
       off += cnt;
     }
+  }
+  if (t->recipe) {
+    // blocked kernel order: prefixes grouped by their last index l (stable, lexicographic within a
+    // group), each followed by its rows q = p + e_i, i = l..n-1 (blocked.cu)
+    const int d = m - 2, P = t->P;
+    t->porder = new (std::nothrow) uint32_t[P];
+    t->gcnt = new (std::nothrow) uint32_t[n];
+    t->qperm = new (std::nothrow) uint32_t[Q];
+    uint32_t* tup = new (std::nothrow) uint32_t[(size_t)P * (d > 0 ? d : 1)];
+    if (!t->porder || !t->gcnt || !t->qperm || !tup) { delete[] tup; general_destroy(t); return nullptr; }
+    int T[kGenMaxM] = {};
+    for (int pi = 0; pi < P; ++pi) {                      // degree-d tuples in lexicographic order (Fig. 4)
+      for (int k = 0; k < d; ++k) tup[(size_t)pi * d + k] = (uint32_t)T[k];
+      int k2 = d - 1;
+      while (k2 >= 0 && T[k2] == n - 1) --k2;
+      if (k2 < 0) break;
+      T[k2] += 1;
+      for (int r = k2 + 1; r < d; ++r) T[r] = T[k2];
+    }
+    int np = 0, nq = 0;
+    for (int l = 0; l < n; ++l) {
+      t->gcnt[l] = 0;
+      for (int pi = 0; pi < P; ++pi) {
+        if ((int)t->plast[pi] != l) continue;
+        t->porder[np++] = (uint32_t)pi;
+        ++t->gcnt[l];
+        for (int i = l; i < n; ++i) {
+          int C[kGenMaxM];
+          for (int k = 0; k < d; ++k) C[k] = (int)tup[(size_t)pi * d + k];
+          C[d] = i;
+          t->qperm[nq++] = (uint32_t)lex_rank(C, m - 1, n);
+        }
+      }
+    }
+    delete[] tup;
+    if (np != P || nq != Q) { general_destroy(t); return nullptr; }
   }
   t->paper_flops = (long long)(m + 2) * U + (long long)(m + 1) * n * Q + 5LL * n;
   // executed per update: per class ~ (m suffix + m prefix + 3 per unique index) + lambda/shift/normalise
@@ -447,6 +490,11 @@ void general_destroy(GeneralTables* t) {
   delete[] t->recipe;
   delete[] t->coef;
   delete[] t->cls;
+  delete[] t->cls_idx;
+  delete[] t->plast;
+  delete[] t->porder;
+  delete[] t->gcnt;
+  delete[] t->qperm;
   delete t;
 }
 
@@ -539,14 +587,27 @@ static int general2_solve(const GeneralTables* t, int64_t N, const float* d_entr
 int general_solve(const GeneralTables* t, int64_t N, const float* d_entries, int S, const float* d_starts, float alpha,
                   float tol, int maxit, float* d_lambda, float* d_x, int32_t* d_iters, uint8_t* d_conv,
                   const sshopm_solve_opts* opts, cudaStream_t st) {
-  if (t->recipe && !(opts && opts->schedule == 4)) {           // item-per-lane kernel unless forced off
-    const int tables = (t->L + t->Q + t->Q * t->n + t->U) * 4;
-    const int per_warp = 32 * (t->U + t->L) * 4;
-    int warps = (200 * 1024 - tables) / per_warp;
-    if (warps > 8) warps = 8;
-    if (warps >= 1)
+  // kernel choice: opts->schedule 3 = item per lane (general2), 5 = blocked (warp per tensor, blocked.cu),
+  // 4 = block per tensor (the paper's mapping); default: blocked (measured faster than the item-per-lane
+  // kernel on every uncompiled shape tried, 2.4x at (7,3) to 33x at (4,10): profiles/r1/large_shapes.txt),
+  // else item per lane, else block per tensor
+  const int sched = opts ? opts->schedule : 0;
+  if (sched == 5 || sched == 0 || sched == 3) {
+    int warps2 = 0, smem2 = 0;
+    if (t->recipe && t->gen2) {
+      const int tables = (t->L + t->Q + t->Q * t->n + t->U) * 4;
+      const int per_warp = 32 * (t->U + t->L) * 4;
+      warps2 = (200 * 1024 - tables) / per_warp;
+      if (warps2 > 8) warps2 = 8;
+      smem2 = tables + warps2 * per_warp;
+    }
+    const bool use2 = warps2 >= 1 && (sched == 3 || (sched == 0 && !blocked_fits(t)));
+    if (use2)
       return general2_solve(t, N, d_entries, S, d_starts, alpha, tol, maxit, d_lambda, d_x, d_iters, d_conv, opts, st,
-                            warps, tables + warps * per_warp);
+                            warps2, smem2);
+    if (sched != 3 && blocked_fits(t))
+      return blocked_solve(t, N, d_entries, S, d_starts, alpha, tol, maxit, d_lambda, d_x, d_iters, d_conv, opts, st);
+    if (sched == 5) return SSHOPM_EUNSUPPORTED;
   }
   const int block = 128;
   const int smem = general_smem(t, block, true);

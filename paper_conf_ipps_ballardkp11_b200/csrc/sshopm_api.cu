@@ -235,7 +235,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const Launchers* L = h->L;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
-  if (opts && (opts->schedule < 0 || opts->schedule > 4)) return SSHOPM_EINVAL;
+  if (opts && (opts->schedule < 0 || opts->schedule > 5)) return SSHOPM_EINVAL;
   if (!L || (opts && opts->schedule >= 3)) {                     // table-driven general kernel (any (m, n))
     if (!h->gen) return SSHOPM_EUNSUPPORTED;
     int rc = general_solve(h->gen, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,

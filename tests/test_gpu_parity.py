@@ -368,10 +368,11 @@ def test_general_apply_exact(dev, m, n):
 
 @pytest.mark.parametrize("m,n,V,alpha", [(5, 4, 24, 4.0), (6, 4, 16, 0.5), (3, 6, 16, 3.0), (10, 2, 32, 0.5), (4, 8, 8, 0.0),
                                          (6, 5, 6, 0.5), (3, 9, 8, 1.0)])
-@pytest.mark.parametrize("schedule", [0, 4])
+@pytest.mark.parametrize("schedule", [0, 3, 4, 5])
 def test_general_solve_parity(dev, m, n, V, alpha, schedule):
-    """(m, n) without a compiled kernel: item-per-lane general kernel (default; n = 9 takes its
-    16-wide register variant) and the block-per-tensor one (schedule 4) vs the oracle."""
+    """(m, n) without a compiled kernel vs the oracle: the default choice, the item-per-lane general
+    kernel (3; n = 9 takes its 16-wide register variant), the block-per-tensor one (4) and the
+    blocked warp-per-tensor one (5)."""
     ent = syn.gen_voxels(m, n, 0, V, 3) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 3)
     st = syn.gen_starts(64, n, 1)
     gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 200, schedule=schedule)
@@ -394,6 +395,55 @@ def test_general_item_kernel_shift_modes(dev, shift):
     if shift == "auto_max":   # convex shift: lambda_k nondecreasing, so lambda_K >= lambda_0 = A x0^m
         lam0 = _solve(dev, m, n, ent, st, shift, -1.0, 0, schedule=3)[0]
         assert np.all(a[0] >= lam0 - 1e-4 * np.maximum(1, np.abs(lam0)))
+
+
+# ------------------------------------------------------- blocked kernel (8(f) row 4) --
+@pytest.mark.parametrize("m,n,V,S,alpha", [(2, 5, 40, 64, 2.0), (3, 4, 33, 100, 1.5), (4, 3, 50, 128, 0.0),
+                                           (4, 10, 6, 32, 0.0), (6, 6, 5, 48, 0.5), (5, 7, 7, 16, 3.0),
+                                           (4, 3, 9, 300, 0.5)])
+def test_blocked_solve_parity(dev, m, n, V, S, alpha):
+    """Blocked warp-per-tensor kernel (schedule 5) vs the oracle: m = 2 (empty prefix) and m = 3
+    (prefix = x), a compiled shape forced onto it, larger shapes ((4,10): U = 715, (6,6): U = 462),
+    S < 32 (a tensor cannot fill the warp), S > 256 and ragged tensor counts (buffer hand-over)."""
+    ent = syn.gen_voxels(m, n, 0, V, 5) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 5)
+    st = syn.gen_starts(S, n, 4)
+    gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 300, schedule=5)
+    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 300, gpu), 0.05)
+
+
+@pytest.mark.parametrize("shift", ["auto_max", "auto_min", "per_tensor"])
+def test_blocked_shift_modes_match_item_kernel(dev, shift):
+    """Blocked kernel with per-tensor and automatic shifts: fixed-K (tol < 0) lambda_K agrees with the
+    item-per-lane general kernel (same arithmetic, same shift) and iteration counts are exact."""
+    m, n, V, S = 5, 4, 37, 100
+    ent = syn.gen_uniform_tensors(m, n, V, 13)
+    st = syn.gen_starts(S, n, 6)
+    alpha = shift
+    if shift == "per_tensor":   # alternating convex / concave shifts of the R17 bound: contractive runs
+        from oracle import sshopm as OR
+        sgn = np.where(np.arange(V) % 2 == 0, 1.0, -1.0)
+        alpha = torch.from_numpy((sgn * OR.convexity_shift(ent, m, n)).astype(np.float32)).to(dev)
+    a = _solve(dev, m, n, ent, st, alpha, -1.0, 40, schedule=5)
+    b = _solve(dev, m, n, ent, st, alpha, -1.0, 40, schedule=3)
+    assert np.all(a[2] == 40) and np.all(b[2] == 40) and not a[3].any()
+    assert np.all(np.abs(a[0] - b[0]) <= 1e-4 * np.maximum(1, np.abs(b[0])))
+
+
+def test_blocked_total_iters_and_tiny(dev):
+    """Blocked kernel: the device iteration counter equals sum(iters); V = 1 and S = 1 work."""
+    m, n = 6, 6
+    for V, S in [(1, 1), (1, 40), (3, 1)]:
+        ent = syn.gen_voxels(m, n, 0, V, 8)
+        st = syn.gen_starts(S, n, 9)
+        s = sh.Solver(m, n)
+        ti = torch.zeros(1, dtype=torch.int64, device=dev)
+        lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.5, 1e-6, 300,
+                                 schedule=5, total_iters=ti)
+        torch.cuda.synchronize()
+        assert int(ti.item()) == int(it.sum().item())
+        rl, rx, ri, rc = O.sshopm(ent, st, m, n, 0.5, 1e-6, 300)
+        both = (cv.cpu().numpy() == 1) & rc
+        assert np.all(np.abs(lam.cpu().numpy()[both] - rl[both]) <= 1e-4 * np.maximum(1, np.abs(rl[both])))
 
 
 # ------------------------------------------------------------ classification --
