@@ -226,6 +226,10 @@ def main():
         else:
             dist.init_process_group("gloo")
     m, n, S, Nloc = cfg["m"], cfg["n"], cfg["S"], cfg["N"]
+    strong = bool(cfg.get("total")) and not a.voxels     # C5: fixed whole volume split over the ranks
+    if strong:
+        assert Nloc % world == 0, "strong-scaling config: tensors must divide evenly over the ranks"
+        Nloc //= world
     solver = sh.Solver(m, n)
     U = solver.U
 
@@ -401,13 +405,21 @@ def main():
     Fe = Fx - Fu                                                          # monomials + 2*T1 + lambda
     alg_flops = Fx * iters_local + Fe * Nloc * S
     achieved = alg_flops * a.steps / (solve_ms / 1e3) / 1e12             # rank-local solve kernel
-    traffic = fma_pct = None
+    traffic = fma_pct = exec_gflop = None
     tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tf):
         with open(tf) as fh:
             prof = json.load(fh)
         traffic = prof.get(a.config)
         fma_pct = prof.get(a.config + "_fma_pipe_active_pct")
+        exec_gflop = prof.get(a.config + "_executed_fp32_gflop")
+    # SURVEY 8(d) metrics 6-7 from the last step's outputs (outside the timed region): converged
+    # fraction, dedup cluster histogram, executed-flop fraction (ncu count / this run's solve time),
+    # voxel-solves/s against the peak-equivalent rate peak / (F_paper x mean iters x S)
+    conv_frac = float(cv.float().mean().item())
+    counts = torch.cat([blk[1][0] for blk in blocks]).to(torch.int64)
+    hist = torch.bincount(counts.clamp(max=KMAX + 1), minlength=KMAX + 2).cpu().tolist()
+    mean_it = iters_all / (Nloc * world * S)
     cpu = None
     if world == 1 and not a.no_cpu:
         nv = a.cpu_voxels or (16384 if (m, n) == (4, 3) else 512)
@@ -418,8 +430,8 @@ def main():
                "voxel_solves_per_s": r["voxel_solves_per_s"]}
     line = {
         "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
-        "ms_per_step": tot_ms / a.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "f32", "data": "synthetic",
+        "ms_per_step": tot_ms / a.steps, "higher_is_better": True, "scaling": "strong" if strong else "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": a.config, "m": m, "n": n, "tensors_per_gpu": Nloc, "tensors_total": Nloc * world,
                    "starts": S, "alpha": cfg["alpha"], "tol": cfg["tol"], "maxit": cfg["maxit"],
                    "dedup": {"lam_tol": LAM_TOL, "ang_tol": ANG_TOL, "kmax": KMAX},
@@ -430,7 +442,10 @@ def main():
                                    f"(chunk i gathered while chunk i+1 solves)" if world > 1 else "")},
         "voxel_solves_per_s": vps,
         "start_solves_per_s": vps * S,
-        "mean_iters": iters_all / (Nloc * world * S),
+        "mean_iters": mean_it,
+        "converged_frac": conv_frac,
+        "dedup_clusters_hist": {str(k) if k <= KMAX else f">{KMAX}": v for k, v in enumerate(hist)},
+        "voxel_solves_frac_of_peak_equiv": vps / (peak_tflops * 1e12 / (F * mean_it * S)),
         "ms_solve_per_step": solve_ms / a.steps,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tflops, "unit": "TFLOP/s",
                      "frac": achieved / peak_tflops, "traffic": traffic,
@@ -439,6 +454,8 @@ def main():
                      "flops_per_update": Fx, "flops_lambda0_eval": Fe,
                      "flops_per_launch": alg_flops,
                      "fma_pipe_active_pct_ncu": fma_pct,
+                     "executed_frac_ncu": (exec_gflop * 1e9 / (solve_ms / a.steps / 1e3) / 1e12 / peak_tflops
+                                           if exec_gflop and world == 1 else None),
                      "flops_note": "algorithmic FP32 flops per launch = flops_per_update x sum(iters) + flops_lambda0_eval x N*S "
                                    "(update: monomials + 2*T1 + lambda + shift + norm + scale; lambda_0: monomials + 2*T1 + lambda; DESIGN.md 7)"},
         "cpu_baseline": cpu,

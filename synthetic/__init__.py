@@ -131,5 +131,8 @@ CONFIGS = {
     "C3": dict(m=6, n=3, N=1 << 20, S=128, alpha=0.25, tol=1e-6, maxit=100),
     "C4a": dict(m=8, n=3, N=1 << 18, S=128, alpha=0.5, tol=1e-6, maxit=100),
     "C4b": dict(m=4, n=6, N=1 << 18, S=128, alpha=0.0, tol=1e-6, maxit=100),
-    "C5": dict(m=4, n=3, N=1 << 23, S=128, alpha=0.0, tol=1e-6, maxit=100),
+    # C5: N is the whole volume, sharded over the ranks (strong scaling); the others are per rank
+    "C5": dict(m=4, n=3, N=1 << 23, S=128, alpha=0.0, tol=1e-6, maxit=100, total=True),
+    # SURVEY 8(d) extra: C2 at alpha = 0.5, the paper-like iteration load (~17.8 updates per solve)
+    "C2a": dict(m=4, n=3, N=1 << 20, S=128, alpha=0.5, tol=1e-6, maxit=100),
 }
