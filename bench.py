@@ -54,6 +54,9 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-voxels", type=int, default=0)
     ap.add_argument("--e2e-chunk", type=int, default=0, help="tensors per run_host chunk (0: auto)")
+    ap.add_argument("--e2e-rep", action="store_true",
+                    help="e2e also returns each cluster's representative start (default: the SURVEY 8(e) record "
+                         "count | K x (lambda, x, mult), 84 B per tensor for (4,3), K = 4)")
     ap.add_argument("--gather-chunks", type=int, default=0,
                     help="N > 1: solve+dedup the rank's range in C chunks and gather chunk i on a side stream "
                          "while chunk i+1 solves (0: 4 when N > 1, else 1)")
@@ -361,8 +364,9 @@ def main():
         outs = {"count": torch.empty(Nloc, dtype=torch.int32).pin_memory(),
                 "lambda": torch.empty((Nloc, KMAX), dtype=torch.float32).pin_memory(),
                 "x": torch.empty((Nloc, KMAX, n), dtype=torch.float32).pin_memory(),
-                "mult": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory(),
-                "rep": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()}
+                "mult": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()}
+        if a.e2e_rep:                                     # representative start per cluster (diagnostic)
+            outs["rep"] = torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()
         chunk = a.e2e_chunk or min(65536, max(4096, Nloc // 16))   # the library default (host_pipeline.cu)
         solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
                         chunk_tensors=chunk, out=outs)

@@ -302,7 +302,8 @@ class Solver:
 
     def run_host(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, lam_tol=1e-2, ang_tol=0.05, kmax=8,
                  raw=False, chunk_tensors=0, out=None):
-        """End-to-end on HOST arrays (numpy or pinned CPU torch tensors); returns a dict of host arrays."""
+        """End-to-end on HOST arrays (numpy or pinned CPU torch tensors); returns a dict of host arrays.
+        A caller-provided `out` without "rep" skips the representative-start field (d_out_rep = NULL)."""
         def ptr(a):
             if hasattr(a, "data_ptr"):
                 if not a.is_contiguous():
@@ -326,7 +327,8 @@ class Solver:
         tot = ctypes.c_ulonglong(0)
         _check(lib().sshopm_run_host(self._h, N, ptr(entries), S, ptr(starts), float(alpha), float(tol), int(maxit),
                                      float(lam_tol), float(ang_tol), int(kmax), ptr(out["count"]), ptr(out["lambda"]),
-                                     ptr(out["x"]), ptr(out["mult"]), ptr(out["rep"]), *rawp, int(chunk_tensors),
+                                     ptr(out["x"]), ptr(out["mult"]), ptr(out["rep"]) if out.get("rep") is not None else None,
+                                     *rawp, int(chunk_tensors),
                                      ctypes.byref(tot)), "sshopm_run_host")
         out["total_iters"] = tot.value
         return out

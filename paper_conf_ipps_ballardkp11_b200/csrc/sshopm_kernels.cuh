@@ -69,10 +69,16 @@ struct Shape {
   static constexpr int NX = (N + 1) / 2;    // float2 slots holding x
   static constexpr int QP = Q / 2;          // q-pairs of the odd output (leftover q handled scalar)
   // B-form keeps Q*N coefficient-folded entries per lane; raw form keeps U.
-  static constexpr bool BFORM = (Q * N <= 64);   // (8,3) B-form (108 words, 186 regs) measured slower: 7.5 vs 6.3 ms
+#ifndef SSHOPM_BFORM_MAX
+#define SSHOPM_BFORM_MAX 64
+#endif
+#ifndef SSHOPM_RAW_MINB_SMALL
+#define SSHOPM_RAW_MINB_SMALL 2
+#endif
+  static constexpr bool BFORM = (Q * N <= SSHOPM_BFORM_MAX);   // (8,3) B-form (108 words, 186 regs) measured slower: 7.5 vs 6.3 ms
   static constexpr int PW_B = Q * NP * 2 + (ODD ? 2 * QP + (Q % 2) : 0);
   static constexpr int PW = round4(BFORM ? PW_B : U);   // packed words per tensor
-  static constexpr int MINB = BFORM ? (Q * N <= 32 ? 4 : (Q * N <= 64 ? 2 : 1)) : (U <= 48 ? 2 : 1);
+  static constexpr int MINB = BFORM ? (Q * N <= 32 ? 4 : (Q * N <= 64 ? 2 : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
 };
 
 // ---------------------------------------------------------- pack kernel ----
