@@ -23,8 +23,9 @@
 //     previous one (no per-tensor tail);
 //   * the dimension n is a template parameter, so x, g and the inner i / j
 //     loops of a block are registers and unrolled code; the prefix monomials
-//     x^p (degree m-2, any m) are built per step from their own prefixes in
-//     lane-interleaved shared memory (bank-conflict free), as in general.cu.
+//     x^p (degree m-2, any m) are x^{p - e_l} x_l with x_l a register (l is
+//     compile-time in the grouped loop), so only degrees 1..m-3 are built per
+//     step, in lane-interleaved shared memory (bank-conflict free).
 // Stopping rule, shift, degenerate cases and outputs are those of every other
 // kernel (readings R1-R7); results match the oracle under the same contract.
 #include <cstdio>
@@ -43,7 +44,8 @@ struct BlkParams {
   const float* coef;         // [Q] (m-1)!/q!
   const uint32_t* cls;       // [Q][n] class(q + e_j)
   const int* cls_mult;       // [U] m!/k! (automatic shift)
-  const uint32_t* pidx;      // [P] degree-(m-2) prefixes grouped by last index (stable)
+  const uint32_t* pidx;      // [P] per degree-(m-2) prefix p (grouped by last index l, stable): the
+                             //     index of p - e_l among the stored monomials (m >= 4)
   const uint32_t* gcnt;      // [n] prefixes per last index
   const uint32_t* qperm;     // [Q] B-row order (per grouped prefix p: q = p + e_i, i = last(p)..n-1)
   float* out_lambda;
@@ -55,8 +57,8 @@ struct BlkParams {
   unsigned int* counter;     // tensor counter (zeroed by the host)
   long long N;
   int m, U, S, L, Q, P;
-  int low;                   // lane-private monomials of degree 1..m-2 (L - Q; mono[0..n) = x)
-  int mono_words;            // per-lane shared words: max(low, n)
+  int low;                   // monomials of degree 1..m-2 in the recipe (L - Q)
+  int mono_words;            // per-lane shared words: degrees 1..m-3 (mono[0..n) = x), at least n
   int buf_words;             // words of one B buffer (Q * round4(n), + 4 for the buffer's shift)
   float alpha, tol;
   int alpha_mode, maxit, refill_k;
@@ -123,7 +125,7 @@ __global__ void __launch_bounds__(128) sshopm_blocked_kernel(const BlkParams p) 
   __syncthreads();
 
   const int m = p.m, S = p.S, Q = p.Q, P = p.P, low = p.low;
-  const int offP = low - (m >= 3 ? P : 0);                         // first prefix monomial (degree m-2 >= 1)
+  const int offP = low - (m >= 3 ? P : 0);                         // stored monomials: degree 1..m-3 = [0, offP)
   // warp-uniform: tensor held by each buffer (-1: none), the buffer being filled and its next start
   long long bt0 = -1, bt1 = -1;
   int fb = 1, fill_s = S;
@@ -207,7 +209,7 @@ __global__ void __launch_bounds__(128) sshopm_blocked_kernel(const BlkParams p) 
     }
 
     // ---- one SS-HOPM step (Fig. 1) ----
-    for (int i = N; i < low; ++i) {                                 // prefixes of degree 2..m-2
+    for (int i = N; i < offP; ++i) {                                // monomials of degree 2..m-3
       const uint32_t r = t_rec[i];
       MONO(i) = MONO(r & 0xffffu) * MONO(r >> 16);
     }
@@ -221,10 +223,12 @@ __global__ void __launch_bounds__(128) sshopm_blocked_kernel(const BlkParams p) 
 #pragma unroll
     for (int l = 0; l < N; ++l) {
       const int cnt = (int)t_gcnt[l];
-      float mpn = (m >= 3 && cnt > 0) ? MONO(offP + (int)t_pidx[pp]) : 1.f;
+      // x^p = x^{p - e_l} x_l: the prefix's own prefix from shared memory (prefetched one block
+      // ahead), x_l from a register (l is compile-time here); m = 3: x^p = x_l, m = 2: x^p = 1
+      float mpn = (m >= 4 && cnt > 0) ? MONO((int)t_pidx[pp]) : 1.f;
       for (int c = 0; c < cnt; ++c, ++pp) {
-        const float mp = mpn;                                       // prefetched: x^p of this block
-        if (m >= 3 && c + 1 < cnt) mpn = MONO(offP + (int)t_pidx[pp + 1]);
+        const float mp = (m >= 4) ? mpn * x[l] : (m == 3 ? x[l] : 1.f);
+        if (m >= 4 && c + 1 < cnt) mpn = MONO((int)t_pidx[pp + 1]);
 #pragma unroll
         for (int i = l; i < N; ++i) {
           const float cm = mp * x[i];
@@ -271,7 +275,8 @@ static int blk_smem(const GeneralTables* t, int warps) {
   const int NP4 = (t->n + 3) / 4 * 4;
   const int tab_words = (t->L + t->P + t->n + 3) / 4 * 4;
   const int bw = (t->Q * NP4 + 4 + 3) / 4 * 4;
-  const int mono = t->L - t->Q > t->n ? t->L - t->Q : t->n;
+  const int stored = t->L - t->Q - (t->m >= 3 ? t->P : 0);           // degrees 1..m-3
+  const int mono = stored > t->n ? stored : t->n;
   return 4 * (tab_words + warps * (2 * bw + 4 + 32 * mono));
 }
 
@@ -332,7 +337,7 @@ int blocked_solve(const GeneralTables* t, int64_t N, const float* d_entries, int
   if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.coef, t->coef, (size_t)t->Q * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.cls, t->cls_idx, (size_t)t->Q * n * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.cls_mult, t->mult, (size_t)t->U * 4, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.pidx, t->porder, (size_t)t->P * 4, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.pidx, t->ppar, (size_t)t->P * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.gcnt, t->gcnt, (size_t)n * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync((void*)p.qperm, t->qperm, (size_t)t->Q * 4, cudaMemcpyHostToDevice, st);
   if (e != cudaSuccess) { cudaFreeAsync(tab, st); return cuda_fail(e, "blocked: table upload"); }
@@ -352,7 +357,8 @@ int blocked_solve(const GeneralTables* t, int64_t N, const float* d_entries, int
   p.Q = t->Q;
   p.P = t->P;
   p.low = t->L - t->Q;
-  p.mono_words = p.low > n ? p.low : n;
+  const int stored = p.low - (t->m >= 3 ? t->P : 0);
+  p.mono_words = stored > n ? stored : n;
   p.buf_words = t->Q * ((n + 3) / 4 * 4) + 4;
   p.alpha = alpha;
   p.tol = tol;

@@ -476,6 +476,11 @@ GeneralTables* general_create(int m, int n) {
     }
     delete[] tup;
     if (np != P || nq != Q) { general_destroy(t); return nullptr; }
+    t->ppar = new (std::nothrow) uint32_t[P];
+    if (!t->ppar) { general_destroy(t); return nullptr; }
+    const long long offP = (L - Q) - P;                  // recipe index of the first degree-(m-2) monomial
+    for (int k = 0; k < P; ++k)
+      t->ppar[k] = m >= 4 ? (t->recipe[offP + t->porder[k]] & 0xffffu) : 0u;
   }
   t->paper_flops = (long long)(m + 2) * U + (long long)(m + 1) * n * Q + 5LL * n;
   // executed per update: per class ~ (m suffix + m prefix + 3 per unique index) + lambda/shift/normalise
@@ -493,6 +498,7 @@ void general_destroy(GeneralTables* t) {
   delete[] t->cls_idx;
   delete[] t->plast;
   delete[] t->porder;
+  delete[] t->ppar;
   delete[] t->gcnt;
   delete[] t->qperm;
   delete t;
@@ -589,7 +595,7 @@ int general_solve(const GeneralTables* t, int64_t N, const float* d_entries, int
                   const sshopm_solve_opts* opts, cudaStream_t st) {
   // kernel choice: opts->schedule 3 = item per lane (general2), 5 = blocked (warp per tensor, blocked.cu),
   // 4 = block per tensor (the paper's mapping); default: blocked (measured faster than the item-per-lane
-  // kernel on every uncompiled shape tried, 2.4x at (7,3) to 33x at (4,10): profiles/r1/large_shapes.txt),
+  // kernel on every uncompiled shape tried, 2x at (5,4) to 47x at (4,10): profiles/r1/large_shapes.txt),
   // else item per lane, else block per tensor
   const int sched = opts ? opts->schedule : 0;
   if (sched == 5 || sched == 0 || sched == 3) {

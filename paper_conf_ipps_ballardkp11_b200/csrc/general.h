@@ -29,6 +29,7 @@ struct GeneralTables {           // host copies; uploaded per call (handles own 
   int P = 0;                     // degree-(m-2) monomials (1 for m = 2: the empty prefix)
   uint32_t* plast = nullptr;     // [P] their last (largest) index, lexicographic order
   uint32_t* porder = nullptr;    // [P] prefixes grouped by last index (stable)
+  uint32_t* ppar = nullptr;      // [P] for porder[k]: recipe index of its own prefix p - e_last (m >= 4; else 0)
   uint32_t* gcnt = nullptr;      // [n] prefixes per last index
   uint32_t* qperm = nullptr;     // [Q] B-row order: for p in porder, q = p + e_i for i = last(p)..n-1
 };
