@@ -60,6 +60,9 @@ def parse():
     ap.add_argument("--gather-chunks", type=int, default=0,
                     help="N > 1: solve+dedup the rank's range in C chunks and gather chunk i on a side stream "
                          "while chunk i+1 solves (0: 4 when N > 1, else 1)")
+    ap.add_argument("--gather", default="nccl", choices=["nccl", "p2p"],
+                    help="N > 1: A9 as NCCL gathers per chunk (default), or p2p: the dedup kernel stores the records "
+                         "straight into rank 0's buffer over NVLink (IPC-mapped peer memory, no collective)")
     ap.add_argument("--dump-records", default="", help="rank 0: save the gathered dedup records (.npz) after the run")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process group backend for N > 1 (gloo: exercise the multi-rank path on one GPU)")
@@ -252,8 +255,13 @@ def main():
     n_chunks = a.gather_chunks or (4 if world > 1 else 1)
     bounds = SH.chunk_bounds(Nloc, n_chunks)
     n_chunks = len(bounds)
-    rec = torch.empty(SH.chunked_record_words(Nloc, n_chunks, KMAX, n)[0], dtype=torch.int32, device=dev)
-    blocks = SH.chunked_record_views(rec, Nloc, n_chunks, KMAX, n)
+    peer = None
+    if world > 1 and a.gather == "p2p":
+        peer = SH.PeerRecords(Nloc, n_chunks, KMAX, n, rank, world, dev)
+        blocks = peer.blocks                              # this rank's slice of rank 0's buffer
+    else:
+        rec = torch.empty(SH.chunked_record_words(Nloc, n_chunks, KMAX, n)[0], dtype=torch.int32, device=dev)
+        blocks = SH.chunked_record_views(rec, Nloc, n_chunks, KMAX, n)
     titers = torch.zeros(1, dtype=torch.int64, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
@@ -282,7 +290,7 @@ def main():
                                total_iters=ti, schedule=a.schedule, fused=a.fused)
             if ev is not None:
                 ev[1].record(stream)
-        if world > 1:
+        if world > 1 and peer is None:
             gather(c)
 
     def gather(c):
@@ -298,7 +306,7 @@ def main():
     def run_path(count_iters=False, evs=None):
         for c in range(n_chunks):
             run_chunk(c, count_iters, None if evs is None else evs[c])
-        if world > 1:
+        if world > 1 and peer is None:
             stream.wait_stream(side)                      # the step ends when the last gather has landed
 
     def step(count_iters=False):
@@ -349,8 +357,13 @@ def main():
     else:
         solve_ms, iters_all = float(stats[2]), float(stats[1])
 
+    if a.dump_records and world > 1 and peer is not None:
+        torch.cuda.synchronize()
+        dist.barrier()                                    # every rank's dedup stores have landed in rank 0's buffer
     if a.dump_records and rank == 0:
-        if world > 1:
+        if world > 1 and peer is not None:
+            merged = peer.merged()
+        elif world > 1:
             merged = SH.merge_chunked(gathered, Nloc, n_chunks, KMAX, n)
         else:
             merged = SH.merge_chunked([[blk] for blk, _ in blocks], Nloc, n_chunks, KMAX, n)
@@ -390,6 +403,9 @@ def main():
 
     if rank != 0:
         if world > 1:
+            if peer is not None:
+                dist.barrier()                            # rank 0 unmaps last
+                peer.close()
             dist.destroy_process_group()
         return
 
@@ -442,8 +458,10 @@ def main():
                    "flop_count": "paper-style F_paper(m,n) x sum(iters), reading R12",
                    "l2": "flushed between timed steps (512 MiB write outside the events)",
                    "parallelism": f"tensor-range shards x{world}" +
-                                  (f" + {a.backend.upper()} gather of dedup records in {n_chunks} chunks "
-                                   f"(chunk i gathered while chunk i+1 solves)" if world > 1 else "")},
+                                  ((" + dedup records stored by the dedup kernel into rank 0's memory over "
+                                    "peer mappings (p2p, no collective)") if world > 1 and peer is not None else
+                                   (f" + {a.backend.upper()} gather of dedup records in {n_chunks} chunks "
+                                    f"(chunk i gathered while chunk i+1 solves)" if world > 1 else ""))},
         "voxel_solves_per_s": vps,
         "start_solves_per_s": vps * S,
         "mean_iters": mean_it,
@@ -470,6 +488,9 @@ def main():
     }
     print(json.dumps(line), flush=True)
     if world > 1:
+        if peer is not None:
+            dist.barrier()
+            peer.close()
         dist.destroy_process_group()
 
 

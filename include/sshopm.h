@@ -215,6 +215,22 @@ int sshopm_launch_count(sshopm_t h, int64_t* count);
 const char* sshopm_status_string(int code);
 const char* sshopm_last_cuda_error(void);
 
+/* Peer memory for the multi-GPU record gather.  Rank 0 allocates
+ * the gather buffer here and exports it; every other rank maps it and passes pointers into it as
+ * sshopm_dedup's outputs, so the dedup kernel's record stores travel over NVLink straight into rank 0's
+ * memory: the gather is fused into the kernel that produces the records (no separate collective).
+ *   sshopm_ipc_alloc: cudaMalloc of `bytes` on the current device (the one allocation this library
+ *     hands out; free it with sshopm_ipc_free); *d_ptr receives it and h_handle (host, caller-owned,
+ *     SSHOPM_IPC_HANDLE_BYTES) the opaque handle other processes of this node pass to sshopm_ipc_import.
+ *   sshopm_ipc_import: maps such a handle into this process (peer access enabled lazily); *d_ptr is
+ *     the buffer's device address here.  Map once, reuse; sshopm_ipc_release unmaps it.
+ * Errors: EINVAL (null arguments, bytes == 0), ENOMEM, ECUDA (the runtime refused: e.g. no P2P path). */
+#define SSHOPM_IPC_HANDLE_BYTES 64
+int sshopm_ipc_alloc(size_t bytes, void** d_ptr, void* h_handle);
+int sshopm_ipc_free(void* d_ptr);
+int sshopm_ipc_import(const void* h_handle, void** d_ptr);
+int sshopm_ipc_release(void* d_ptr);
+
 /* Comma-separated list of (m,n) pairs compiled into this build, e.g. "2x3,4x3". */
 const char* sshopm_supported_shapes(void);
 

@@ -69,6 +69,10 @@ def lib():
         "sshopm_status_string": (ctypes.c_char_p, [I]),
         "sshopm_last_cuda_error": (ctypes.c_char_p, []),
         "sshopm_supported_shapes": (ctypes.c_char_p, []),
+        "sshopm_ipc_alloc": (I, [ctypes.c_size_t, ctypes.POINTER(P), P]),
+        "sshopm_ipc_free": (I, [P]),
+        "sshopm_ipc_import": (I, [P, ctypes.POINTER(P)]),
+        "sshopm_ipc_release": (I, [P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -85,6 +89,48 @@ def _status(code):
 def _check(code, where):
     if code != OK:
         raise SSHOPMError(code, where)
+
+
+IPC_HANDLE_BYTES = 64
+
+
+def ipc_alloc(nbytes):
+    """Device buffer other processes of this node can map: -> (device address, handle bytes)."""
+    p = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+    _check(lib().sshopm_ipc_alloc(ctypes.c_size_t(int(nbytes)), ctypes.byref(p), h), "sshopm_ipc_alloc")
+    return int(p.value), h.raw
+
+
+def ipc_free(ptr):
+    _check(lib().sshopm_ipc_free(ctypes.c_void_p(ptr)), "sshopm_ipc_free")
+
+
+def ipc_import(handle):
+    """Map another process's exported allocation; returns its device address (int)."""
+    p = ctypes.c_void_p()
+    _check(lib().sshopm_ipc_import(ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES), ctypes.byref(p)),
+           "sshopm_ipc_import")
+    return int(p.value)
+
+
+def ipc_release(ptr):
+    _check(lib().sshopm_ipc_release(ctypes.c_void_p(ptr)), "sshopm_ipc_release")
+
+
+class _CudaArray:
+    """__cuda_array_interface__ wrapper: lets torch alias a raw device address without a copy."""
+
+    def __init__(self, ptr, shape, typestr):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr, "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
+def device_view(ptr, shape, dtype, device):
+    """A torch tensor aliasing `ptr` (e.g. a peer buffer mapped by ipc_import); no copy."""
+    torch = _torch()
+    ts = {torch.int32: "<i4", torch.float32: "<f4", torch.uint8: "|u1"}[dtype]
+    return torch.as_tensor(_CudaArray(ptr, shape, ts), device=device)
 
 
 def supported_shapes():

@@ -148,6 +148,43 @@ const char* sshopm_status_string(int code) {
 
 const char* sshopm_last_cuda_error(void) { return g_last_cuda_error; }
 
+int sshopm_ipc_alloc(size_t bytes, void** d_ptr, void* h_handle) {
+  static_assert(sizeof(cudaIpcMemHandle_t) == SSHOPM_IPC_HANDLE_BYTES, "IPC handle size");
+  if (!d_ptr || !h_handle || bytes == 0) return SSHOPM_EINVAL;
+  *d_ptr = nullptr;
+  cudaError_t e = cudaMalloc(d_ptr, bytes);
+  if (e == cudaErrorMemoryAllocation) { cudaGetLastError(); return SSHOPM_ENOMEM; }
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_ipc_alloc");
+  cudaIpcMemHandle_t hd;
+  e = cudaIpcGetMemHandle(&hd, *d_ptr);
+  if (e != cudaSuccess) { cudaFree(*d_ptr); *d_ptr = nullptr; return cuda_fail(e, "sshopm_ipc_alloc: handle"); }
+  memcpy(h_handle, &hd, sizeof(hd));
+  return SSHOPM_OK;
+}
+
+int sshopm_ipc_free(void* d_ptr) {
+  if (!d_ptr) return SSHOPM_EINVAL;
+  cudaError_t e = cudaFree(d_ptr);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_ipc_free");
+  return SSHOPM_OK;
+}
+
+int sshopm_ipc_import(const void* h_handle, void** d_ptr) {
+  if (!h_handle || !d_ptr) return SSHOPM_EINVAL;
+  cudaIpcMemHandle_t hd;
+  memcpy(&hd, h_handle, sizeof(hd));
+  cudaError_t e = cudaIpcOpenMemHandle(d_ptr, hd, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_ipc_import");
+  return SSHOPM_OK;
+}
+
+int sshopm_ipc_release(void* d_ptr) {
+  if (!d_ptr) return SSHOPM_EINVAL;
+  cudaError_t e = cudaIpcCloseMemHandle(d_ptr);
+  if (e != cudaSuccess) return cuda_fail(e, "sshopm_ipc_release");
+  return SSHOPM_OK;
+}
+
 const char* sshopm_supported_shapes(void) {
   static const char* s =
 #define SHAPE(mm, nn) #mm "x" #nn ","

@@ -116,3 +116,44 @@ def merge_chunked(gathered, n_per_rank, n_chunks, kmax, n):
             b = b.cpu().numpy() if hasattr(b, "cpu") else np.asarray(b)
             parts.append(tuple(v[:v1 - v0] for v in record_views(b, per, kmax, n)))
     return tuple(np.concatenate([p[i] for p in parts], axis=0) for i in range(5))
+
+
+class PeerRecords:
+    """Rank 0's gather buffer, mapped into every rank through the library's IPC entry points
+    (sshopm_ipc_alloc / sshopm_ipc_import): rank r passes views of its own slice as sshopm_dedup's
+    outputs, so the dedup kernel stores its records over NVLink straight into rank 0's memory — the
+    gather is fused into the producing kernel.  Layout: [world][chunked record
+    buffer of one rank] (chunked_record_words), so merge_chunked reassembles it like gathered blocks."""
+
+    def __init__(self, n_per_rank, n_chunks, kmax, n, rank, world, device):
+        import torch
+        import torch.distributed as dist
+        import paper_conf_ipps_ballardkp11_b200 as sh
+        self.rank, self.world, self.n_chunks, self.kmax, self.n = rank, world, n_chunks, kmax, n
+        self.n_per_rank = n_per_rank
+        self.words, _ = chunked_record_words(n_per_rank, n_chunks, kmax, n)
+        obj = [None]
+        if rank == 0:
+            self.ptr, handle = sh.ipc_alloc(4 * self.words * world)
+            obj = [handle]
+        if world > 1:
+            dist.broadcast_object_list(obj, src=0)
+        if rank != 0:
+            self.ptr = sh.ipc_import(obj[0])
+        self.buf = sh.device_view(self.ptr, (world * self.words,), torch.int32, device)
+        self.slices = [self.buf[r * self.words:(r + 1) * self.words] for r in range(world)]
+        self.blocks = chunked_record_views(self.slices[rank], n_per_rank, n_chunks, kmax, n)
+
+    def merged(self):
+        """Rank 0, after every rank's kernels finished (barrier): global records in tensor order."""
+        gathered = [[chunked_record_views(self.slices[r], self.n_per_rank, self.n_chunks, self.kmax, self.n)[c][0]
+                     for r in range(self.world)] for c in range(len(self.blocks))]
+        return merge_chunked(gathered, self.n_per_rank, self.n_chunks, self.kmax, self.n)
+
+    def close(self):
+        import paper_conf_ipps_ballardkp11_b200 as sh
+        self.buf = self.slices = self.blocks = None
+        if self.rank == 0:
+            sh.ipc_free(self.ptr)
+        else:
+            sh.ipc_release(self.ptr)

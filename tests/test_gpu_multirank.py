@@ -37,9 +37,12 @@ def test_bench_two_ranks_gloo():
     assert d["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
 
 
-def test_chunked_gather_bitwise_equal_to_one_process(tmp_path):
+@pytest.mark.parametrize("gather", ["nccl", "p2p"])
+def test_chunked_gather_bitwise_equal_to_one_process(tmp_path, gather):
     """C5 invariant: dedup records gathered from P = 2 ranks, each solving its range in
-    3 chunks, equal bit for bit those of one process solving the whole volume in one call."""
+    3 chunks, equal bit for bit those of one process solving the whole volume in one call — through the
+    collective (gloo stands in for NCCL on one GPU) and through peer memory (the dedup kernel of rank 1
+    storing into rank 0's IPC-mapped buffer)."""
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
@@ -51,7 +54,7 @@ def test_chunked_gather_bitwise_equal_to_one_process(tmp_path):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"),
            "--gpus", "2", "--steps", "1", "--warmup", "3", "--backend", "gloo", "--no-cpu", "--no-e2e",
-           "--voxels", str(nloc), "--gather-chunks", "3", "--dump-records", dump]
+           "--voxels", str(nloc), "--gather-chunks", "3", "--dump-records", dump, "--gather", gather]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
     assert r.returncode == 0, r.stderr[-2000:]
     got = np.load(dump)
