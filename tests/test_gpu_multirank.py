@@ -37,23 +37,23 @@ def test_bench_two_ranks_gloo():
     assert d["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
 
 
-@pytest.mark.parametrize("gather", ["nccl", "p2p"])
-def test_chunked_gather_bitwise_equal_to_one_process(tmp_path, gather):
-    """C5 invariant: dedup records gathered from P = 2 ranks, each solving its range in
-    3 chunks, equal bit for bit those of one process solving the whole volume in one call — through the
-    collective (gloo stands in for NCCL on one GPU) and through peer memory (the dedup kernel of rank 1
-    storing into rank 0's IPC-mapped buffer)."""
+@pytest.mark.parametrize("world,gather", [(2, "nccl"), (2, "p2p"), (4, "nccl"), (4, "p2p")])
+def test_chunked_gather_bitwise_equal_to_one_process(tmp_path, world, gather):
+    """C5 invariant: dedup records gathered from P = 2 and 4 ranks, each solving its range
+    in 3 chunks, equal bit for bit those of one process solving the whole volume in one call — through the
+    collective (gloo stands in for NCCL on one GPU) and through peer memory (the dedup kernels of ranks
+    1..P-1 storing into rank 0's IPC-mapped buffer)."""
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     import numpy as np
     import paper_conf_ipps_ballardkp11_b200 as sh
     import synthetic as syn
-    nloc, kmax = 8192, 4
+    nloc, kmax = 16384 // world, 4
     dump = str(tmp_path / "rec.npz")
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(world),
            "--master-addr", "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"),
-           "--gpus", "2", "--steps", "1", "--warmup", "3", "--backend", "gloo", "--no-cpu", "--no-e2e",
+           "--gpus", str(world), "--steps", "1", "--warmup", "3", "--backend", "gloo", "--no-cpu", "--no-e2e",
            "--voxels", str(nloc), "--gather-chunks", "3", "--dump-records", dump, "--gather", gather]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
     assert r.returncode == 0, r.stderr[-2000:]
@@ -61,7 +61,7 @@ def test_chunked_gather_bitwise_equal_to_one_process(tmp_path, gather):
     cfg = syn.CONFIGS["C2"]
     m, n, S = cfg["m"], cfg["n"], cfg["S"]
     dev = torch.device("cuda:0")
-    ent = torch.from_numpy(syn.gen_voxels(m, n, 0, 2 * nloc, seed=0)).to(dev)
+    ent = torch.from_numpy(syn.gen_voxels(m, n, 0, world * nloc, seed=0)).to(dev)
     st = torch.from_numpy(syn.gen_starts(S, n, seed=0)).to(dev)
     solver = sh.Solver(m, n)
     lam, x, it, cv = solver.solve(ent, st, cfg["alpha"], cfg["tol"], cfg["maxit"])
