@@ -78,7 +78,10 @@ struct Shape {
   static constexpr bool BFORM = (Q * N <= SSHOPM_BFORM_MAX);   // (8,3) B-form (108 words, 186 regs) measured slower: 7.5 vs 6.3 ms
   static constexpr int PW_B = Q * NP * 2 + (ODD ? 2 * QP + (Q % 2) : 0);
   static constexpr int PW = round4(BFORM ? PW_B : U);   // packed words per tensor
-  static constexpr int MINB = BFORM ? (Q * N <= 32 ? 4 : (Q * N <= 64 ? 2 : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
+#ifndef SSHOPM_BFORM32_MINB
+#define SSHOPM_BFORM32_MINB 4
+#endif
+  static constexpr int MINB = BFORM ? (Q * N <= 32 ? SSHOPM_BFORM32_MINB : (Q * N <= 64 ? 2 : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
 };
 
 // ---------------------------------------------------------- pack kernel ----
