@@ -18,7 +18,7 @@ import synthetic as syn  # noqa: E402
 from tests import parity as PR  # noqa: E402
 
 # config -> number of sampled tensors checked against the oracle
-SAMPLES = {"C2": 512, "C3": 192, "C4a": 32, "C4b": 128}
+SAMPLES = {"C2": 512, "C2a": 384, "C3": 192, "C4a": 32, "C4b": 128}
 
 
 @pytest.fixture(scope="module")
@@ -28,7 +28,7 @@ def dev():
     return torch.device("cuda:0")
 
 
-@pytest.mark.parametrize("cfg_name", ["C2", "C3", "C4a", "C4b"])
+@pytest.mark.parametrize("cfg_name", ["C2", "C2a", "C3", "C4a", "C4b"])
 def test_fullsize_sampled_parity(dev, cfg_name):
     c = syn.CONFIGS[cfg_name]
     m, n, N, S = c["m"], c["n"], c["N"], c["S"]
@@ -54,4 +54,31 @@ def test_fullsize_sampled_parity(dev, cfg_name):
     assert rep["flag_unexplained"] == 0, rep
     assert rep["lam_unexplained"] == 0, rep
     assert rep["angle_unexplained"] == 0, rep
-    assert rep["sensitive_frac"] <= 1e-3, rep
+    # C2a (alpha = 0.5) converges slowly, so more lanes end at the stopping boundary, where FP32 / FP64
+    # rounding decides the flag (measured: 76 of 49,152 sampled lanes, all at the boundary, 60 of them
+    # also witness-sensitive): DESIGN.md P0 caps explained lanes at 0.5% there, 0.1% elsewhere
+    assert rep["sensitive_frac"] <= (5e-3 if cfg_name == "C2a" else 1e-3), rep
+
+
+@pytest.mark.parametrize("m,n,N,alpha,k", [(4, 10, 16384, 0.0, 24), (6, 6, 16384, 0.5, 16)])
+def test_blocked_default_sampled_parity(dev, m, n, N, alpha, k):
+    """Larger shapes through the default table-driven path (the blocked kernel) at the size
+    tools/large_shapes.py times: every-lane properties, and a spread sample of tensors vs the oracle."""
+    ent = syn.gen_voxels(m, n, 0, N, seed=0)
+    st = syn.gen_starts(128, n, seed=0)
+    solver = sh.Solver(m, n)
+    lam, x, it, cv = solver.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), alpha, 1e-6, 100)
+    torch.cuda.synchronize()
+    nx = torch.linalg.vector_norm(x, dim=2)
+    assert float((nx - 1).abs().max()) < 5e-6
+    assert int(it.min()) >= 0 and int(it.max()) <= 100
+    assert float((cv == 1).float().mean()) > 0.95
+    idx = np.unique(np.linspace(0, N - 1, k).astype(np.int64))
+    sel = torch.from_numpy(idx).to(dev)
+    gpu = tuple(t.index_select(0, sel).cpu().numpy() for t in (lam, x, it, cv))
+    rep = PR.solve_parity(ent[idx], st, m, n, alpha, 1e-6, 100, gpu)
+    print((m, n), {kk: v for kk, v in rep.items() if kk != "details"})
+    assert rep["flag_unexplained"] == 0, rep
+    assert rep["lam_unexplained"] == 0, rep
+    assert rep["angle_unexplained"] == 0, rep
+    assert rep["sensitive_frac"] <= 0.02, rep
