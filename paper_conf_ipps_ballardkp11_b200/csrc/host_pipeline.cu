@@ -9,6 +9,7 @@
 // Device buffers and streams are cached in the handle (HostCache) and reused
 // across calls — allocation, not transfer, would otherwise dominate; calls on
 // one handle serialise on the cache mutex.  sshopm_destroy frees the cache.
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -125,12 +126,25 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     }
     c->chunk = chunk;
   }
+  static const bool ramp = [] { const char* v = getenv("SSHOPM_RAMP"); return !(v && v[0] == '0'); }();
   CK(cudaMemcpyAsync(c->d_starts, h_starts, sizeof(float) * S * n, cudaMemcpyHostToDevice, c->slots[0].st), "run_host: H2D");
   CK(cudaMemsetAsync(c->d_total, 0, sizeof(unsigned long long), c->slots[0].st), "run_host: memset");
   CK(cudaStreamSynchronize(c->slots[0].st), "run_host: sync");
-  for (long long c0 = 0, ci = 0; c0 < N; c0 += chunk, ++ci) {
+  for (long long c0 = 0, ci = 0, cn = 0; c0 < N; c0 += cn, ++ci) {
     Slot& s = c->slots[ci % kSlots];
-    const long long cn = (N - c0 < chunk) ? (N - c0) : chunk;
+    // ramped chunk sizes: chunk/4, chunk/2 first and last, so the exposed pipeline fill (first H2D) and
+    // drain (last dedup + D2H) are short; full chunks in between (SSHOPM_RAMP=0 disables)
+    const long long left = N - c0;
+    cn = chunk;
+    if (ramp && N > 4 * chunk) {
+      const long long q = chunk / 4;
+      if (ci == 0) cn = q;                                   // ramp up: chunk/4, chunk/2, chunk, ...
+      else if (ci == 1) cn = 2 * q;
+      else if (left > chunk + 2 * q) cn = chunk < left - 3 * q ? chunk : left - 3 * q;   // leave >= 3/4 chunk
+      else if (left > 2 * q) cn = left - q;                 // ... and end on a quarter chunk
+    }
+    if (cn < 1) cn = 1;
+    if (cn > left) cn = left;
     CK(cudaMemcpyAsync(s.ent, h_entries + c0 * U, sizeof(float) * cn * U, cudaMemcpyHostToDevice, s.st), "run_host: H2D");
     sshopm_solve_opts o;
     memset(&o, 0, sizeof(o));
