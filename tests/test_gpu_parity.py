@@ -110,22 +110,30 @@ def test_fixed_k(dev, alpha, K):
     assert r["unexplained"] == 0, r
 
 
-def test_special_cases(dev):
-    """maxit = 0 -> (lam_0, x_0); zero start -> 0; odd S, N not a multiple of anything."""
-    m, n = 4, 3
-    ent = syn.gen_voxels(m, n, 0, 37, 0)
+@pytest.mark.parametrize("m,n,schedule", [(4, 3, 0), (4, 3, 5), (4, 3, 3), (5, 4, 0)])
+def test_special_cases(dev, m, n, schedule):
+    """maxit = 0 -> (lam_0, x_0); zero start -> 0; odd S, N not a multiple of anything — for the
+    unrolled kernel, the blocked (5) and item-per-lane (3) table-driven kernels, and a shape without
+    a compiled kernel (default: blocked)."""
+    ent = syn.gen_voxels(m, n, 0, 37, 0) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, 37, 0)
+    alpha = 0.0 if m % 2 == 0 else 2.0
     st = syn.gen_starts(13, n, 0)
     st[4] = 0.0
-    lam, x, it, cv = _solve(dev, m, n, ent, st, 0.0, 1e-6, 0)
+    lam, x, it, cv = _solve(dev, m, n, ent, st, alpha, 1e-6, 0, schedule=schedule)
     assert (it == 0).all() and not cv.any()
     x0 = O.normalise_starts(st)
     assert np.allclose(x, np.broadcast_to(x0, x.shape), atol=1e-7)
     full = O.expand_full(ent, m, n)
     lam0 = O.axm(np.repeat(full, 13, 0), np.tile(x0, (37, 1))).reshape(37, 13)
     assert np.allclose(lam, lam0, atol=1e-5)
-    lam, x, it, cv = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
+    lam, x, it, cv = _solve(dev, m, n, ent, st, alpha, 1e-6, 100, schedule=schedule)
     assert (lam[:, 4] == 0).all() and (x[:, 4] == 0).all() and (it[:, 4] == 0).all() and not cv[:, 4].any()
-    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, (lam, x, it, cv)))
+    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 100, (lam, x, it, cv)), 0.05 if m % 2 else 1e-3)
+    # N = 0 is a no-op
+    s = sh.Solver(m, n)
+    out = s.solve(torch.zeros((0, ent.shape[1]), device=dev), torch.from_numpy(st).to(dev), alpha, 1e-6, 100,
+                  schedule=schedule)
+    assert all(t.shape[0] == 0 for t in out)
 
 
 def test_invariance_across_launch_configs(dev):
