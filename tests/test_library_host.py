@@ -104,3 +104,17 @@ def test_general_shapes_tables(m, n):
     assert np.array_equal(s.class_index(), np.array(O.class_list(m, n), dtype=np.int32))
     assert s.paper_flops_per_iter == O.paper_flops_per_iter(m, n)
     s.close()
+
+
+def test_ipc_entry_points_reject_bad_arguments():
+    """Peer-memory gather entry points (multi-GPU A9): argument checks happen before any CUDA call."""
+    L = sh.lib()
+    p = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(sh.IPC_HANDLE_BYTES)
+    assert L.sshopm_ipc_alloc(0, ctypes.byref(p), h) == sh.EINVAL
+    assert L.sshopm_ipc_alloc(1024, None, h) == sh.EINVAL
+    assert L.sshopm_ipc_alloc(1024, ctypes.byref(p), None) == sh.EINVAL
+    assert L.sshopm_ipc_import(None, ctypes.byref(p)) == sh.EINVAL
+    assert L.sshopm_ipc_import(h, None) == sh.EINVAL
+    assert L.sshopm_ipc_free(None) == sh.EINVAL
+    assert L.sshopm_ipc_release(None) == sh.EINVAL
