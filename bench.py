@@ -63,6 +63,9 @@ def parse():
     ap.add_argument("--gather", default="nccl", choices=["nccl", "p2p"],
                     help="N > 1: A9 as NCCL gathers per chunk (default), or p2p: the dedup kernel stores the records "
                          "straight into rank 0's buffer over NVLink (IPC-mapped peer memory, no collective)")
+    ap.add_argument("--graph", action="store_true",
+                    help="N = 1: capture one step (pack, solve, dedup launches) in a CUDA graph and replay it "
+                         "(launch-bound small volumes); the solve is then timed together with the step")
     ap.add_argument("--dump-records", default="", help="rank 0: save the gathered dedup records (.npz) after the run")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process group backend for N > 1 (gloo: exercise the multi-rank path on one GPU)")
@@ -320,6 +323,23 @@ def main():
     torch.cuda.synchronize()
     iters_local = int(titers.item())
 
+    graph = None
+    if a.graph:
+        assert world == 1, "--graph is for N = 1"
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream(device=dev)
+        cap.wait_stream(stream)
+        with torch.cuda.stream(cap):
+            run_path()                                    # warm the capture stream (workspaces, caches)
+            cap.synchronize()
+            lc0 = solver.launch_count()
+            with torch.cuda.graph(graph, stream=cap):
+                run_path()
+            launches_per_replay = solver.launch_count() - lc0
+        stream.wait_stream(cap)
+        torch.cuda.synchronize()
+
     def tev():
         return torch.cuda.Event(enable_timing=True)
     ev = [(tev(), tev()) for _ in range(a.steps)]
@@ -335,16 +355,25 @@ def main():
             flush.zero_()
             e0, e2 = ev[i]
             e0.record(stream)
-            run_path(evs=cev[i])
+            if graph is not None:
+                graph.replay()
+                cev[i][0][0].record(stream)               # no solve-only window inside a graph
+                cev[i][0][1].record(stream)
+            else:
+                run_path(evs=cev[i])
             e2.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     launches = solver.launch_count() - l0
+    if graph is not None:
+        launches = launches_per_replay * a.steps          # kernels inside each replayed graph
     t_step = [e0.elapsed_time(e2) for e0, e2 in ev]
     # pack + solve kernels of every chunk (with --solve-dedup: the whole call)
     t_solve = [sum(s0.elapsed_time(s1) for s0, s1 in cs) for cs in cev]
+    if graph is not None:
+        t_solve = t_step                                  # roofline over the whole replayed step (conservative)
     tot_ms = float(sum(t_step))
     cdev = dev if a.backend == "nccl" else torch.device("cpu")
     stats = torch.tensor([tot_ms, float(iters_local), float(sum(t_solve))], dtype=torch.float64, device=cdev)
@@ -457,6 +486,7 @@ def main():
                    "dedup": {"lam_tol": LAM_TOL, "ang_tol": ANG_TOL, "kmax": KMAX},
                    "flop_count": "paper-style F_paper(m,n) x sum(iters), reading R12",
                    "l2": "flushed between timed steps (512 MiB write outside the events)",
+                   "cuda_graph": bool(graph is not None),
                    "parallelism": f"tensor-range shards x{world}" +
                                   ((" + dedup records stored by the dedup kernel into rank 0's memory over "
                                     "peer mappings (p2p, no collective)") if world > 1 and peer is not None else
