@@ -219,6 +219,39 @@ struct Coefs {
 
   // g = A x^{M-1} from the Q monomials mq.
   __device__ __forceinline__ void contract(const float (&mq)[S::Q], float2 (&gp)[S::NP > 0 ? S::NP : 1], float& gs) const {
+#ifndef SSHOPM_PAIRED_CONTRACT
+    // small rows: scalar FFMA, q outer / j inner (the monomial is the operand every output of a q shares,
+    // reused from the operand cache); measured faster than the FFMA2 forms below on B200 for (4,3)
+    // (C2 solve 4.43 -> 4.32 ms, C2a 7.41 -> 7.25) but slower for (6,3) (C3 11.98 -> 12.14):
+    // profiles/r1/solve_variants.txt.  Outputs g_j as independent chains; the odd last output sequential.
+    if constexpr (BF && S::Q * N <= 30) {
+      constexpr int base = S::Q * S::NP * 2;
+      float g[N];
+      static_for<S::Q>([&](auto qq) {
+        constexpr int q = decltype(qq)::value;
+        static_for<S::NP>([&](auto pp) {
+          constexpr int p = decltype(pp)::value;
+          if constexpr (q == 0) {
+            g[2 * p] = word<(q * S::NP + p) * 2>() * mq[q];
+            g[2 * p + 1] = word<(q * S::NP + p) * 2 + 1>() * mq[q];
+          } else {
+            g[2 * p] = fmaf(word<(q * S::NP + p) * 2>(), mq[q], g[2 * p]);
+            g[2 * p + 1] = fmaf(word<(q * S::NP + p) * 2 + 1>(), mq[q], g[2 * p + 1]);
+          }
+        });
+        if constexpr (S::ODD) {
+          if constexpr (q == 0) g[N - 1] = word<base>() * mq[0];
+          else g[N - 1] = fmaf(word<base + q>(), mq[q], g[N - 1]);
+        }
+      });
+      static_for<S::NP>([&](auto pp) {
+        constexpr int p = decltype(pp)::value;
+        gp[p] = f2(g[2 * p], g[2 * p + 1]);
+      });
+      if constexpr (S::ODD) gs = g[N - 1];
+      return;
+    }
+#endif
     if constexpr (BF) {
       static_for<S::NP>([&](auto pp) {
         constexpr int p = decltype(pp)::value;
@@ -298,6 +331,7 @@ __device__ __forceinline__ void monomials(const float2 (&xs)[(N + 1) / 2], float
 template <int M, int N>
 struct X21 { static constexpr bool v = (M == 4 && N == 3); };
 
+#ifndef SSHOPM_SCALAR_MONO
 template <>
 __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
   const float2 x01 = xs[0], x21 = xs[1];
@@ -313,6 +347,7 @@ __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&m
   mq[0] = m01.x; mq[1] = m01.y; mq[2] = m23.x; mq[3] = m23.y; mq[4] = m45.x;
   mq[5] = m45.y; mq[6] = m67.x; mq[7] = m67.y; mq[8] = m89.x; mq[9] = m89.y;
 }
+#endif
 
 // g = A x^{M-1} (pairs gp, odd tail gs) and lambda = x . g
 template <int M, int N>
