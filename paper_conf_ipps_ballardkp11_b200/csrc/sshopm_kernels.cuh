@@ -426,7 +426,8 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
       xs[1] = f2(hp[1].x * r, xs[0].y);
     } else {
 #pragma unroll
-      for (int i = 0; i < S::NX; ++i) xs[i] = __fmul2_rn(hp[i], bc(r));
+      for (int i = 0; i < S::NP; ++i) xs[i] = __fmul2_rn(hp[i], bc(r));
+      if constexpr (S::ODD) xs[S::NX - 1].x = hp[S::NX - 1].x * r;   // .y stays 0
     }
     lamp = lam;
     ++k;
