@@ -377,7 +377,9 @@ __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&
 // Stopped lanes freeze (x, lambda_prev, k unchanged) so a frozen lane
 // recomputes bit-identical values until the warp refills it.
 // SHIFT: 0 alpha = 0, 1 alpha > 0, 2 alpha < 0 (alpha passed negated), 3 per-lane (la = |alpha|, ls = sign)
-template <int M, int N, int SHIFT>
+// KIDLE: lanes without an item hold k = INT_MAX (>= maxit), so the maxit test also stops them and the
+// per-step stop predicate needs no separate `has` term (schedule 1 keeps this convention).
+template <int M, int N, int SHIFT, bool KIDLE = false>
 __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[Shape<M, N>::NX], float& lam,
                                             float& lamp, int& k, bool& conv, bool& stop, bool has, float alpha,
                                             float la, float ls, float tol, int maxit) {
@@ -415,7 +417,8 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
     nn = t.x + t.y;
   }
   const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
-  stop = (!has) | conv | (k >= maxit) | deg;                  // non-short-circuit: one predicate chain
+  if constexpr (KIDLE) stop = conv | (k >= maxit) | deg;      // idle lanes: k = INT_MAX
+  else stop = (!has) | conv | (k >= maxit) | deg;             // non-short-circuit: one predicate chain
   const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
   // the freeze is a guarded update that ptxas if-converts into predicated
   // FMUL2 / FMUL / MOV / IADD: no select per component (+9% step throughput
@@ -606,7 +609,7 @@ sshopm_solve_kernel(const SolveParams p) {
         for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
         if constexpr (XL) xs[1].y = v[1];                  // (x2, x1) layout
       }
-      k = ok ? 0 : k;
+      k = ok ? 0 : (stop ? 0x7fffffff : k);                  // idle lanes: k >= maxit keeps them stopped
       lamp = ok ? __int_as_float(0x7fffffff) : lamp;         // NaN: the first test never fires (reading R2)
       has = stop ? ok : has;
       if (!exhausted) {
@@ -657,7 +660,7 @@ sshopm_solve_kernel(const SolveParams p) {
     // ---------------- SS-HOPM steps (Fig. 1), STEPS per refill check ----------------
 #pragma unroll
     for (int rep = 0; rep < STEPS; ++rep)
-      sshopm_step<M, N, SHIFT>(cf, xs, lam, lamp, k, conv, stop, has, alpha, la, ls, tol, maxit);
+      sshopm_step<M, N, SHIFT, true>(cf, xs, lam, lamp, k, conv, stop, has, alpha, la, ls, tol, maxit);
     __syncwarp();
   }
 
