@@ -354,6 +354,10 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   p.chunk_tensors = chunk_tensors;
   p.S = S;
   p.divS = make_fastdiv((uint32_t)S);
+  p.s_log2 = -1;
+  if ((S & (S - 1)) == 0)
+    for (int b = 0; b < 31; ++b)
+      if ((1 << b) == S) p.s_log2 = b;
   p.alpha = alpha;
   p.alpha_t = ws.alpha_t;
   p.tol = tol;

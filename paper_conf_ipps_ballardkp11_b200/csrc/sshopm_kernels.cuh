@@ -452,6 +452,7 @@ struct SolveParams {
   int chunk_tensors;         // tensors per chunk
   int S;
   FastDiv divS;
+  int s_log2;                // log2(S) if S is a power of two, else -1
   float alpha, tol;
   const float* alpha_t;      // SHIFT == 3: per-tensor shift [N] (from the pack kernel)
   int maxit;
@@ -589,16 +590,24 @@ sshopm_solve_kernel(const SolveParams p) {
       const bool ok = stop && !exhausted && (cur || t < n_end);
       if (ok) {
         const Idx v0 = cur ? c_vox : n_vox;
-        const uint32_t vq = fast_div(t, p.divS);
-        const uint32_t s = t - vq * S_;
         item = v0 * (Idx)S_ + (Idx)t;
+        Idx tv;                                            // tensor of the item
+        uint32_t s;                                        // its start
+        if (p.s_log2 >= 0) {                               // S a power of two (the paper's 128): shift and mask
+          tv = item >> p.s_log2;
+          s = (uint32_t)item & (S_ - 1u);
+        } else {
+          const uint32_t vq = fast_div(t, p.divS);
+          s = t - vq * S_;
+          tv = v0 + (Idx)vq;
+        }
         if constexpr (FUSED) cseq = cur ? cur_seq : claim_seq;
         if constexpr (SHIFT == 3) {
-          const float at = __ldg(p.alpha_t + (v0 + (Idx)vq));
+          const float at = __ldg(p.alpha_t + tv);
           ls = at >= 0.f ? 1.f : -1.f;                     // Fig. 1 lines 2-5 (R5: alpha = 0 -> "+")
           la = fabsf(at);
         }
-        cf.load(p.packed + (v0 + (Idx)vq) * (Idx)(S::PW / 4));
+        cf.load(p.packed + tv * (Idx)(S::PW / 4));
         float v[4 * SST4];
 #pragma unroll
         for (int i = 0; i < SST4; ++i) {
