@@ -168,6 +168,41 @@ __device__ __forceinline__ void step_p(const Coefs<M, N, true>& cf, float2 (&xs)
 // V 0: the kernel's step (B-form, conv test, selects, k);  1: without the stop logic;
 //   3: raw-form contraction (scalar FFMA on class entries);  4: two items per lane sharing the coefficients
 //   5: q-paired contraction;  6: q-paired, lambda_prev unconditional;  7/8: step_v MODE 0/1
+// Two starts per lane vectorised ACROSS starts: every FP op is an FFMA2/FMUL2 on
+// (start A, start B) with the B-form coefficient broadcast; stop logic per start.
+__device__ __forceinline__ void step_x2(const Coefs<M, N, true>& cf, float2 (&X)[3], float2& lamp, float2& lam,
+                                        int& kA, int& kB, bool& sA, bool& sB, float tol, int maxit) {
+  const float2 s00 = __fmul2_rn(X[0], X[0]), s01 = __fmul2_rn(X[0], X[1]), s02 = __fmul2_rn(X[0], X[2]);
+  const float2 s11 = __fmul2_rn(X[1], X[1]), s12 = __fmul2_rn(X[1], X[2]), s22 = __fmul2_rn(X[2], X[2]);
+  const float2 mq[10] = {__fmul2_rn(X[0], s00), __fmul2_rn(X[0], s01), __fmul2_rn(X[0], s02), __fmul2_rn(X[0], s11),
+                         __fmul2_rn(X[0], s12), __fmul2_rn(X[0], s22), __fmul2_rn(X[1], s11), __fmul2_rn(X[1], s12),
+                         __fmul2_rn(X[1], s22), __fmul2_rn(X[2], s22)};
+  constexpr int base = SH::Q * SH::NP * 2;
+  float2 g0, g1, g2;
+  static_for<SH::Q>([&](auto qq) {
+    constexpr int q = decltype(qq)::value;
+    if constexpr (q == 0) {
+      g0 = __fmul2_rn(bc(cf.template word<0>()), mq[0]);
+      g1 = __fmul2_rn(bc(cf.template word<1>()), mq[0]);
+      g2 = __fmul2_rn(bc(cf.template word<base>()), mq[0]);
+    } else {
+      g0 = __ffma2_rn(bc(cf.template word<2 * q>()), mq[q], g0);
+      g1 = __ffma2_rn(bc(cf.template word<2 * q + 1>()), mq[q], g1);
+      g2 = __ffma2_rn(bc(cf.template word<base + q>()), mq[q], g2);
+    }
+  });
+  lam = __ffma2_rn(X[2], g2, __ffma2_rn(X[1], g1, __fmul2_rn(X[0], g0)));
+  const float2 nn = __ffma2_rn(g2, g2, __ffma2_rn(g1, g1, __fmul2_rn(g0, g0)));
+  const float2 r = f2(rsqrt_ftz(nn.x), rsqrt_ftz(nn.y));
+  const bool cA = fabsf(lam.x - lamp.x) <= tol * fmaxf(1.0f, fabsf(lam.x));
+  const bool cB = fabsf(lam.y - lamp.y) <= tol * fmaxf(1.0f, fabsf(lam.y));
+  sA = cA | (kA >= maxit) | !(nn.x >= 1.17549435e-38f);
+  sB = cB | (kB >= maxit) | !(nn.y >= 1.17549435e-38f);
+  const float2 n0 = __fmul2_rn(g0, r), n1 = __fmul2_rn(g1, r), n2 = __fmul2_rn(g2, r);
+  if (!sA) { X[0].x = n0.x; X[1].x = n1.x; X[2].x = n2.x; lamp.x = lam.x; ++kA; }
+  if (!sB) { X[0].y = n0.y; X[1].y = n1.y; X[2].y = n2.y; lamp.y = lam.y; ++kB; }
+}
+
 template <int V, int MINB>
 __global__ void __launch_bounds__(256, MINB) step_kernel(const float4* packed, float* out, int iters, int maxit) {
   const int t = blockIdx.x * blockDim.x + threadIdx.x;
@@ -184,8 +219,12 @@ __global__ void __launch_bounds__(256, MINB) step_kernel(const float4* packed, f
   int k = 0, k2 = 0;
   bool stop = false, stop2 = false;
   const float tol = 0.f;
+  float2 X2[3] = {f2(xs[0].x, xs2[0].x), f2(xs[0].y, xs2[0].y), f2(xs[1].x, xs2[1].x)};
+  float2 lamp_x2 = f2(lamp, lamp2), lam_x2 = f2(0.f, 0.f);
   for (int it = 0; it < iters; ++it) {
-    if constexpr (V == 1) {
+    if constexpr (V == 10) {
+      step_x2(cf, X2, lamp_x2, lam_x2, k, k2, stop, stop2, tol, maxit);
+    } else if constexpr (V == 1) {
       float2 gp[SH::NP];
       float gs = 0.f;
       lam = evaluate<M, N>(cf, xs, gp, gs);
@@ -209,7 +248,8 @@ __global__ void __launch_bounds__(256, MINB) step_kernel(const float4* packed, f
       step<V == 3>(cf, xs, lamp, lam, k, stop, tol, maxit);
     }
   }
-  float o = lam + xs[0].x + (float)k + (stop ? 1.f : 0.f) + lamp;
+  float o = lam + xs[0].x + (float)k + (stop ? 1.f : 0.f) + (V == 10 ? 0.f : lamp);
+  if constexpr (V == 10) o += lam_x2.x + lam_x2.y + X2[0].x + X2[2].y + lamp_x2.x + lamp_x2.y + (float)k2 + (stop2 ? 1.f : 0.f);
   if constexpr (V == 4) o += lam2 + xs2[0].y + (float)k2 + lamp2 + (stop2 ? 1.f : 0.f);
   out[t] = o;
 }
@@ -227,7 +267,7 @@ void run(const char* name, const float4* packed, float* out, int sms, int ctas) 
   cudaEventSynchronize(e1);
   float ms; cudaEventElapsedTime(&ms, e0, e1);
   ms /= 5;
-  const double flops = (V == 4 ? 2 : 1) * 89.0 * iters * (double)grid * 256;
+  const double flops = (V == 4 || V == 10 ? 2 : 1) * 89.0 * iters * (double)grid * 256;
   cudaFuncAttributes fa; cudaFuncGetAttributes(&fa, step_kernel<V, MINB>);
   printf("{\"variant\":\"%s\",\"ctas_per_sm\":%d,\"regs\":%d,\"ms\":%.4f,\"tflops_alg\":%.2f,\"frac_of_74.4\":%.3f}\n",
          name, ctas, fa.numRegs, ms, flops / ms / 1e9, flops / ms / 1e9 / 74.4);
@@ -243,6 +283,10 @@ int main() {
   cudaMemcpy(packed, h.data(), h.size() * 4, cudaMemcpyHostToDevice);
   cudaMalloc(&out, sms * 8 * 256 * 4);
   run<0, 4>("kernel_step", packed, out, sms, 4);
+  run<9, 4>("predicated_update", packed, out, sms, 4);
+  run<10, 4>("two_starts_ffma2_across_starts", packed, out, sms, 4);
+  run<10, 3>("two_starts_ffma2_across_starts", packed, out, sms, 3);
+  run<10, 2>("two_starts_ffma2_across_starts", packed, out, sms, 2);
   run<0, 2>("kernel_step", packed, out, sms, 2);
   run<0, 4>("kernel_step", packed, out, sms, 3);
   run<1, 4>("no_stop_logic", packed, out, sms, 4);
