@@ -209,9 +209,46 @@ def reference_arm(a, cfg, rank, world):
     print(json.dumps(line), flush=True)
 
 
+# ---------------------------------------------------------------- launcher --
+def free_port():
+    import socket
+    with socket.socket(socket.AF_INET, socket.SOCK_STREAM) as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def launch_command(argv, n, port):
+    """torchrun command line that re-runs this script with the same arguments on n local ranks."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + list(argv)
+
+
+def self_launch(a, argv):
+    """`python bench.py --gpus N` (N > 1) outside torchrun: start the N ranks ourselves, one process per
+    GPU, and return their exit status.  Under torchrun (WORLD_SIZE set) the world size must equal --gpus."""
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is not None:
+        if int(world_env) != a.gpus and "--gpus" in " ".join(argv):
+            raise SystemExit(f"bench.py: WORLD_SIZE={world_env} but --gpus {a.gpus}")
+        return None
+    if a.gpus <= 1:
+        return None
+    env = dict(os.environ)
+    # NCCL's communicator-init log (ranks, NVLS / NVLink topology) goes to files, not to the JSON stdout
+    if a.backend == "nccl" and "NCCL_DEBUG" not in env:
+        os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+        env.update(NCCL_DEBUG="INFO", NCCL_DEBUG_SUBSYS="INIT",
+                   NCCL_DEBUG_FILE=os.path.join(ROOT, "gpurun_out", "nccl_init.%h.%p.log"))
+    import subprocess
+    return subprocess.run(launch_command(argv, a.gpus, free_port()), env=env).returncode
+
+
 # ---------------------------------------------------------------- our arm --
 def main():
     a = parse()
+    rc = self_launch(a, sys.argv[1:])
+    if rc is not None:
+        return rc
     cfg = dict(syn.CONFIGS[a.config])
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -525,4 +562,4 @@ def main():
 
 
 if __name__ == "__main__":
-    main()
+    sys.exit(main() or 0)

@@ -113,7 +113,9 @@ typedef struct {
   void* d_workspace;               /* optional caller-owned device workspace, 256-byte aligned, >= sshopm_workspace_size */
   size_t workspace_bytes;          /* its size; a too-small or misaligned workspace returns EINVAL */
   int schedule;                    /* 0 default, 1 = item per lane (warps claim chunks of whole tensors),
-                                      2 = tensor per lane (a lane walks one tensor's starts); results identical.
+                                      2 = tensor per lane (a lane walks one tensor's starts), 6 = item per lane
+                                      with a branch-free predicated refill and one chunk in flight (measured
+                                      slower on B200, kept for comparison); results identical.
                                       Table-driven general kernel (the only path for (m, n) without a compiled
                                       kernel): 5 = blocked (default): warp per tensor, the
                                       tensor's coefficient-folded rows once per warp in shared memory, blocks of
@@ -130,6 +132,8 @@ typedef struct {
                                       converges to local maxima, Kolda-Mayo [1]); 3 = automatic concave shift -(...)
                                       (minima).  Modes 1-3 use schedule 1. */
   const float* d_alpha;            /* alpha_mode 1: per-tensor shifts [N] */
+  int chunk_tensors;               /* schedule 6: tensors per work chunk a warp claims (0 = default:
+                                      up to 1024 items, at least 8 chunks per resident warp) */
 } sshopm_solve_opts;
 
 /* sshopm_solve with options (opts may be NULL).  Launches two kernels on

@@ -17,7 +17,8 @@ import numpy as np
 __all__ = ["Solver", "SSHOPMError", "lib", "supported_shapes", "library_path"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-library_path = os.path.join(_HERE, "_lib", "libsshopm.so")
+# SSHOPM_LIBRARY: load a variant build (tools/ sweeps) instead of the in-tree product library
+library_path = os.environ.get("SSHOPM_LIBRARY") or os.path.join(_HERE, "_lib", "libsshopm.so")
 _LIB = None
 
 OK, EINVAL, EUNSUPPORTED, ECUDA, ENOMEM = 0, 1, 2, 3, 4
@@ -36,7 +37,7 @@ class _Opts(ctypes.Structure):
     _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
                 ("d_total_iters", ctypes.c_void_p), ("d_workspace", ctypes.c_void_p),
                 ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int), ("fuse_dedup", ctypes.c_int),
-                ("alpha_mode", ctypes.c_int), ("d_alpha", ctypes.c_void_p)]
+                ("alpha_mode", ctypes.c_int), ("d_alpha", ctypes.c_void_p), ("chunk_tensors", ctypes.c_int)]
 
 ALPHA_MODES = {"scalar": 0, "per_tensor": 1, "auto_max": 2, "auto_min": 3}
 
@@ -178,7 +179,7 @@ class Solver:
         _check(lib().sshopm_flops_per_iter(h, ctypes.byref(pf), ctypes.byref(ef)), "sshopm_flops_per_iter")
         self.paper_flops_per_iter = pf.value
         self.exec_flops_per_iter = ef.value
-        self._ws = None            # cached device workspace (torch uint8 tensor)
+        self._ws = {}              # (device, stream handle) -> cached device workspace (torch uint8 tensor)
         self._ws_size = {}         # (N, S) -> bytes
 
     def close(self):
@@ -205,13 +206,21 @@ class Solver:
             self._ws_size[key] = b.value
         return self._ws_size[key]
 
-    def _workspace(self, N, S, device):
+    def _workspace(self, N, S, device, stream=None):
+        """Workspace for a call on `stream`: one cached buffer per (device, stream), allocated on that
+        stream, so calls in flight on different streams never share (or free) each other's workspace."""
         need = self.workspace_size(N, S)
-        ws = self._ws
-        if ws is None or ws.device != device or ws.numel() < need:
-            torch = _torch()
-            ws = torch.empty(need + 256, dtype=torch.uint8, device=device)
-            self._ws = ws
+        torch = _torch()
+        st = torch.cuda.current_stream(device) if stream is None else stream
+        key = (str(device), int(st.cuda_stream))
+        ws = self._ws.get(key)
+        if ws is None or ws.numel() < need:
+            with torch.cuda.stream(st):
+                ws = torch.empty(need + 256, dtype=torch.uint8, device=device)
+            old = self._ws.get(key)
+            if old is not None:
+                old.record_stream(st)      # the previous buffer stays alive until the stream's queued work ends
+            self._ws[key] = ws
         base = ws.data_ptr()
         return ctypes.c_void_p((base + 255) // 256 * 256), need
 
@@ -237,7 +246,7 @@ class Solver:
         return c.value
 
     def solve(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, out=None, refill_threshold=0,
-              ctas_per_sm=0, total_iters=None, stream=None, schedule=0):
+              ctas_per_sm=0, total_iters=None, stream=None, schedule=0, chunk_tensors=0):
         """entries [N, U] f32, starts [S, n] f32 (CUDA) -> (lam [N,S], x [N,S,n], iters [N,S] i32, conv [N,S] u8)."""
         torch = _torch()
         N, S = int(entries.shape[0]), int(starts.shape[0])
@@ -252,8 +261,9 @@ class Solver:
         lam, x, it, cv = out
         args = (_dev(lam, torch.float32, (N, S), "out_lambda"), _dev(x, torch.float32, (N, S, self.n), "out_x"),
                 _dev(it, torch.int32, (N, S), "out_iters"), _dev(cv, torch.uint8, (N, S), "out_converged"))
-        wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
+        wsp, wsb = self._workspace(N, S, dev, stream) if N > 0 else (None, 0)
         opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 0)
+        opts.chunk_tensors = int(chunk_tensors)
         alpha = self._alpha_opts(alpha, N, opts)
         if total_iters is not None:
             if total_iters.dtype != torch.int64 or not total_iters.is_cuda or total_iters.numel() != 1:
@@ -261,6 +271,27 @@ class Solver:
             opts.d_total_iters = total_iters.data_ptr()
         _check(lib().sshopm_solve_ex(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit), *args,
                                      ctypes.byref(opts), _stream(stream)), "sshopm_solve")
+        return out
+
+    def solve_plain(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, out=None, stream=None):
+        """The sshopm_solve entry point itself: library defaults, a workspace the library
+        allocates and frees on the stream (cudaMallocAsync), scalar alpha only."""
+        torch = _torch()
+        N, S = int(entries.shape[0]), int(starts.shape[0])
+        pe = _dev(entries, torch.float32, (N, self.U), "entries")
+        ps = _dev(starts, torch.float32, (S, self.n), "starts")
+        dev = entries.device
+        if out is None:
+            out = (torch.empty((N, S), dtype=torch.float32, device=dev),
+                   torch.empty((N, S, self.n), dtype=torch.float32, device=dev),
+                   torch.empty((N, S), dtype=torch.int32, device=dev),
+                   torch.empty((N, S), dtype=torch.uint8, device=dev))
+        lam, x, it, cv = out
+        _check(lib().sshopm_solve(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit),
+                                  _dev(lam, torch.float32, (N, S), "out_lambda"),
+                                  _dev(x, torch.float32, (N, S, self.n), "out_x"),
+                                  _dev(it, torch.int32, (N, S), "out_iters"),
+                                  _dev(cv, torch.uint8, (N, S), "out_converged"), _stream(stream)), "sshopm_solve")
         return out
 
     def solve_dedup(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, lam_tol=1e-2, ang_tol=0.05, kmax=8,
@@ -290,7 +321,7 @@ class Solver:
         dargs = (_dev(c, torch.int32, (N,), "out_count"), _dev(ol, torch.float32, (N, kmax), "out_clambda"),
                  _dev(ox, torch.float32, (N, kmax, self.n), "out_cx"), _dev(om, torch.int32, (N, kmax), "out_mult"),
                  _dev(orp, torch.int32, (N, kmax), "out_rep"))
-        wsp, wsb = self._workspace(N, S, dev) if N > 0 else (None, 0)
+        wsp, wsb = self._workspace(N, S, dev, stream) if N > 0 else (None, 0)
         opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 1 if fused else 0)
         alpha = self._alpha_opts(alpha, N, opts)
         if total_iters is not None:
@@ -350,18 +381,31 @@ class Solver:
                  raw=False, chunk_tensors=0, out=None):
         """End-to-end on HOST arrays (numpy or pinned CPU torch tensors); returns a dict of host arrays.
         A caller-provided `out` without "rep" skips the representative-start field (d_out_rep = NULL)."""
-        def ptr(a):
+        def ptr(a, dtype, shape, name):
+            """Host pointer of `a` after checking dtype, shape and layout (the C ABI reads raw memory)."""
             if hasattr(a, "data_ptr"):
+                torch = _torch()
+                tdt = {np.float32: torch.float32, np.int32: torch.int32, np.uint8: torch.uint8}[dtype]
+                if a.is_cuda:
+                    raise TypeError(f"{name} must be a host (CPU) tensor")
+                if a.dtype != tdt:
+                    raise TypeError(f"{name} must be {tdt}, got {a.dtype}")
+                if tuple(a.shape) != tuple(shape):
+                    raise ValueError(f"{name} must have shape {tuple(shape)}, got {tuple(a.shape)}")
                 if not a.is_contiguous():
-                    raise ValueError("host tensors must be contiguous")
+                    raise ValueError(f"{name}: host tensors must be contiguous")
                 return ctypes.c_void_p(a.data_ptr())
+            if not isinstance(a, np.ndarray):
+                raise TypeError(f"{name} must be a numpy array or a CPU torch tensor")
+            if a.dtype != np.dtype(dtype):
+                raise TypeError(f"{name} must be {np.dtype(dtype)}, got {a.dtype}")
+            if tuple(a.shape) != tuple(shape):
+                raise ValueError(f"{name} must have shape {tuple(shape)}, got {tuple(a.shape)}")
             if not a.flags["C_CONTIGUOUS"]:
-                raise ValueError("host arrays must be C-contiguous")
+                raise ValueError(f"{name}: host arrays must be C-contiguous")
             return ctypes.c_void_p(a.ctypes.data)
 
         N, S = int(entries.shape[0]), int(starts.shape[0])
-        if tuple(entries.shape) != (N, self.U) or tuple(starts.shape) != (S, self.n):
-            raise ValueError("entries must be [N, U] and starts [S, n]")
         if out is None:
             out = {"count": np.empty(N, np.int32), "lambda": np.empty((N, kmax), np.float32),
                    "x": np.empty((N, kmax, self.n), np.float32), "mult": np.empty((N, kmax), np.int32),
@@ -369,11 +413,18 @@ class Solver:
             if raw:
                 out.update({"raw_lambda": np.empty((N, S), np.float32), "raw_x": np.empty((N, S, self.n), np.float32),
                             "raw_iters": np.empty((N, S), np.int32), "raw_converged": np.empty((N, S), np.uint8)})
-        rawp = [ptr(out[k]) if raw else None for k in ("raw_lambda", "raw_x", "raw_iters", "raw_converged")]
+        n, K, f4, i4, u1 = self.n, int(kmax), np.float32, np.int32, np.uint8
+        pe = ptr(entries, f4, (N, self.U), "entries")
+        ps = ptr(starts, f4, (S, n), "starts")
+        rawspec = {"raw_lambda": (f4, (N, S)), "raw_x": (f4, (N, S, n)), "raw_iters": (i4, (N, S)),
+                   "raw_converged": (u1, (N, S))}
+        rawp = [ptr(out[k], *rawspec[k], k) if raw else None for k in rawspec]
+        rp = ptr(out["rep"], i4, (N, K), "rep") if out.get("rep") is not None else None
         tot = ctypes.c_ulonglong(0)
-        _check(lib().sshopm_run_host(self._h, N, ptr(entries), S, ptr(starts), float(alpha), float(tol), int(maxit),
-                                     float(lam_tol), float(ang_tol), int(kmax), ptr(out["count"]), ptr(out["lambda"]),
-                                     ptr(out["x"]), ptr(out["mult"]), ptr(out["rep"]) if out.get("rep") is not None else None,
+        _check(lib().sshopm_run_host(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit),
+                                     float(lam_tol), float(ang_tol), K, ptr(out["count"], i4, (N,), "count"),
+                                     ptr(out["lambda"], f4, (N, K), "lambda"), ptr(out["x"], f4, (N, K, n), "x"),
+                                     ptr(out["mult"], i4, (N, K), "mult"), rp,
                                      *rawp, int(chunk_tensors),
                                      ctypes.byref(tot)), "sshopm_run_host")
         out["total_iters"] = tot.value

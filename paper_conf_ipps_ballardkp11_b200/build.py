@@ -21,9 +21,10 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-BUILD = os.path.join(ROOT, "build")
-LIBDIR = os.path.join(PKG, "_lib")
-LIB = os.path.join(LIBDIR, "libsshopm.so")
+# SSHOPM_BUILD_DIR / SSHOPM_LIB_OUT: build a variant library elsewhere (tools/ sweeps), never over the product .so
+BUILD = os.environ.get("SSHOPM_BUILD_DIR") or os.path.join(ROOT, "build")
+LIB = os.environ.get("SSHOPM_LIB_OUT") or os.path.join(PKG, "_lib", "libsshopm.so")
+LIBDIR = os.path.dirname(LIB)
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
@@ -39,7 +40,8 @@ def nvcc():
 
 def shapes():
     with open(os.path.join(CSRC, "shapes.def")) as f:
-        return [(int(a), int(b)) for a, b in re.findall(r"^SHAPE\((\d+),\s*(\d+)\)", f.read(), re.M)]
+        sh = [(int(a), int(b)) for a, b in re.findall(r"^SHAPE\((\d+),\s*(\d+)\)", f.read(), re.M)]
+    return sh
 
 
 def _newest_source():

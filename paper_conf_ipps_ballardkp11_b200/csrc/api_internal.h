@@ -11,7 +11,7 @@ struct sshopm_ctx {
   const sshopm::Launchers* L;      // compiled (m, n) kernels, or null
   // host-side launch-shape cache (occupancy per non-fused kernel variant, per device); 0 = not computed
   std::atomic<int> occ_dev;
-  std::atomic<int> occ[4][2][3];   // [shift][wide][schedule]
+  std::atomic<int> occ[4][2][6];   // [shift][wide][schedule - 1]
   sshopm::GeneralTables* gen;      // table-driven kernel tables (any (m, n))
   int m, n, U;
   std::atomic<long long> launches;

@@ -85,11 +85,15 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   if (chunk_tensors <= 0) chunk = chunk < 4096 ? 4096 : (chunk > 65536 ? 65536 : chunk);
   if (chunk > N) chunk = N;
 
-  if (!h->hc) {
-    h->hc = new (std::nothrow) HostCache;
-    if (!h->hc) return SSHOPM_ENOMEM;
+  HostCache* c;
+  {
+    // lazy creation under a process-wide lock, so concurrent first calls on one handle create one cache
+    static std::mutex create_mu;
+    std::lock_guard<std::mutex> g(create_mu);
+    if (!h->hc) h->hc = new (std::nothrow) HostCache;
+    c = h->hc;
   }
-  HostCache* c = h->hc;
+  if (!c) return SSHOPM_ENOMEM;
   std::lock_guard<std::mutex> lock(c->mu);
   int dev = 0;
   cudaGetDevice(&dev);

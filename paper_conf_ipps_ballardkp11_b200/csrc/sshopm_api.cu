@@ -114,7 +114,8 @@ int device_sms() {
 // occupancy of a non-fused solve variant, cached in the handle for the current device
 static cudaError_t cached_occupancy(sshopm_ctx* h, int shift, bool wide, int schedule, int* bps) {
   int dev = 0;
-  cudaGetDevice(&dev);
+  const cudaError_t ge = cudaGetDevice(&dev);
+  if (ge != cudaSuccess) return ge;
   if (h->occ_dev.load(std::memory_order_acquire) != dev + 1) {
     for (auto& a : h->occ)
       for (auto& b : a)
@@ -272,8 +273,8 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const Launchers* L = h->L;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
-  if (opts && (opts->schedule < 0 || opts->schedule > 5)) return SSHOPM_EINVAL;
-  if (!L || (opts && opts->schedule >= 3)) {                     // table-driven general kernel (any (m, n))
+  if (opts && (opts->schedule < 0 || opts->schedule > 6)) return SSHOPM_EINVAL;
+  if (!L || (opts && opts->schedule >= 3 && opts->schedule <= 5)) {   // table-driven general kernel (any (m, n))
     if (!h->gen) return SSHOPM_EUNSUPPORTED;
     int rc = general_solve(h->gen, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
                            d_out_converged, opts, st);
@@ -296,10 +297,11 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   if (alpha_mode == 1 && !opts->d_alpha) return SSHOPM_EINVAL;
   const int shift = alpha_mode ? 3 : (alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2));
   const bool wide = (long long)N * S >= (1LL << 31) - (1LL << 20);
-  // schedule: 1 = item per lane (chunks of whole tensors), 2 = tensor per lane
+  // schedule: 1 = item per lane (two-chunk refill, default), 2 = tensor per lane, 6 = item per lane with the
+  // lean predicated refill (C2: 4.33 vs 4.26 ms for schedule 1, profiles/r2/solve_variants.md)
   int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
-  if (schedule != 1 && schedule != 2) return SSHOPM_EINVAL;   // 3 / 4 (general) handled above
-  if (shift == 3) schedule = 1;                                  // per-tensor alpha: schedule 1 only
+  if (schedule != 1 && schedule != 2 && schedule != 6) return SSHOPM_EINVAL;   // 3-5 (general) handled above
+  if (shift == 3 && schedule == 2) schedule = 1;                 // per-tensor alpha: not on schedule 2
   int bps = 0;
   cudaError_t e = cached_occupancy(h, shift, wide, schedule, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
@@ -311,7 +313,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   int smem = 0;
   const bool fregs = dd && S == 128 && ((uintptr_t)d_out_lambda % 16 == 0) && ((uintptr_t)d_out_x % 16 == 0) &&
                      ((uintptr_t)d_out_converged % 4 == 0);
-  if (dd && schedule == 1 && S <= 1024 && opts && opts->fuse_dedup == 1) {
+  if (dd && schedule != 2 && S <= 1024 && opts && opts->fuse_dedup == 1) {
     const int fs = 8 * fused_smem_words(S, L->n, fregs) * 4;
     int fb = 0;
     if (fs <= 200 * 1024 && L->occupancy(shift, wide, schedule, fregs ? 2 : 1, fs, &fb) == cudaSuccess && fb >= bps) {
@@ -319,12 +321,24 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
       smem = fs;
     }
   }
+  if (fused) schedule = 1;                                       // the fused ring lives in the schedule-1 kernel
   if (opts && opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
-  const int chunk_tensors = chunk_tensors_for(S);                  // schedule 1: >= 256 items per chunk
+  if (opts && opts->chunk_tensors < 0) return SSHOPM_EINVAL;
+  int chunk_tensors = chunk_tensors_for(S);                        // schedule 1: >= 256 items per chunk
+  if (schedule == 6) {
+    // lean schedule: chunks of up to 1024 items, at least 8 per resident warp
+    const long long warps = (long long)sms * bps * 8;
+    long long c = N / (warps * 8);
+    const long long cmax = S >= 1024 ? 1 : 1024 / S;
+    if (c > cmax) c = cmax;
+    if (c < 1) c = 1;
+    chunk_tensors = (int)c;
+    if (opts && opts->chunk_tensors > 0) chunk_tensors = opts->chunk_tensors;
+  }
   const long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
   if (n_chunks >= (1LL << 32) - (1LL << 20) || N >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
   long long grid = (long long)sms * bps;
-  if (schedule == 1) {
+  if (schedule != 2) {
     if (grid * 8 > n_chunks) grid = (n_chunks + 7) / 8;
   } else {
     if (grid * 256 > N) grid = (N + 255) / 256;

@@ -25,6 +25,8 @@ cudaError_t occ2(int schedule, int smem, int* bps) {
   } else {
     if (schedule == 2) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_tpl_kernel<M, N, SH, W>, 256, 0);
   }
+  if (schedule == 6 && F == 0)
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_lean_kernel<M, N, SH, W>, 256, 0);
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W, F>, 256, smem);
 }
 template <int SH, bool W>
@@ -50,7 +52,9 @@ cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaS
   if (schedule == 2) {
     if constexpr (SH == 3) return cudaErrorInvalidValue;     // per-tensor alpha: schedule 1 only
     else sshopm_solve_tpl_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
-  } else {
+  } else if (schedule == 6 && F == 0) {                      // lean predicated refill (measured slower, kept)
+    sshopm_solve_lean_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
+  } else {                                                   // schedule 1 (default) or the fused dedup
     if (smem > 48 * 1024) {
       cudaError_t e = cudaFuncSetAttribute(sshopm_solve_kernel<M, N, SH, W, F>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       if (e != cudaSuccess) return e;

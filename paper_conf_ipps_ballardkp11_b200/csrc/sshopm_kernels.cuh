@@ -43,6 +43,29 @@ __device__ __forceinline__ float rsqrt_ftz(float v) {
 __device__ __forceinline__ float2 f2(float a, float b) { return make_float2(a, b); }
 __device__ __forceinline__ float2 bc(float a) { return make_float2(a, a); }
 __device__ __forceinline__ float4 ldg4(const float4* p) { return __ldg(p); }
+// Predicated global accesses as single predicated instructions (no divergent
+// branch / BSSY region around the refill's stores and loads).
+__device__ __forceinline__ void pst(bool p, float* a, float v) {
+  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %0, 0;\n @q st.global.f32 [%1], %2;\n}"
+               :: "r"((int)p), "l"(a), "f"(v) : "memory");
+}
+__device__ __forceinline__ void pst(bool p, int32_t* a, int32_t v) {
+  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %0, 0;\n @q st.global.b32 [%1], %2;\n}"
+               :: "r"((int)p), "l"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void pst(bool p, uint8_t* a, uint32_t v) {
+  asm volatile("{\n .reg .pred q;\n .reg .b16 t;\n setp.ne.b32 q, %0, 0;\n cvt.u16.u32 t, %2;\n @q st.global.b8 [%1], t;\n}"
+               :: "r"((int)p), "l"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void pld4(bool p, const float4* a, float4& v) {
+  asm("{\n .reg .pred q;\n setp.ne.b32 q, %4, 0;\n @q ld.global.nc.v4.f32 {%0, %1, %2, %3}, [%5];\n}"
+      : "+f"(v.x), "+f"(v.y), "+f"(v.z), "+f"(v.w) : "r"((int)p), "l"(a));
+}
+__device__ __forceinline__ unsigned int atom_add1(unsigned int* a) {   // plain (not warp-aggregated) atomic
+  unsigned int r;
+  asm volatile("atom.global.add.u32 %0, [%1], 1;" : "=r"(r) : "l"(a) : "memory");
+  return r;
+}
 
 constexpr int round4(int v) { return (v + 3) / 4 * 4; }
 // SS-HOPM steps per refill check (trip).  More steps amortise the ballot and
@@ -84,6 +107,23 @@ struct Shape {
   static constexpr int MINB = BFORM ? (Q * N <= 32 ? SSHOPM_BFORM32_MINB : (Q * N <= 64 ? 2 : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
 };
 
+// State layout of x (see xget below): slot of component i.
+#ifndef SSHOPM_43_FORM
+#define SSHOPM_43_FORM 2   // (4,3) step: 2 = (x0,x1),(x2,x1) layout, 8 FMUL2 monomials, scalar FFMA contraction (default:
+                           // C2 4.26 ms); 1 = natural layout, (g0,g1) FFMA2 + g2 FFMA (4.44); 0 = X02 layout, scalar (4.43)
+#endif
+template <int M, int N>
+struct X02 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 0); };
+template <int M, int N>
+struct N43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 1); };
+// form 2: the round-1 layout, x held as (x0, x1), (x2, x1) (slot 3 duplicates x1), monomials as 8 FMUL2
+template <int M, int N>
+struct X21 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 2); };
+template <int M, int N>
+__host__ __device__ constexpr int xslot(int i) {
+  return X02<M, N>::v ? (i == 0 ? 0 : (i == 1 ? 2 : 1)) : i;
+}
+
 // ---------------------------------------------------------- pack kernel ----
 // B-form row:  [ (B_{q,2p}, B_{q,2p+1}) for q, p ] [ (B_{2t,N-1}, B_{2t+1,N-1}) for t < QP ] [B_{Q-1,N-1} if Q odd] [0 pad]
 // with B_{q,j} = ((M-1)!/q!) * a_{class(q + e_j)}   (Eq. 6 regrouped by monomial)
@@ -96,7 +136,8 @@ sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float
                    float* __restrict__ alpha_t) {
   using S = Shape<M, N>;
   if (counter && blockIdx.x == 0 && threadIdx.x == 0) { counter[0] = 0u; counter[1] = 0u; }   // solve's chunk / overflow counters
-  // normalised starts x_0 = s / ||s|| in FP32 (reading R7), rows padded to SST floats
+  // normalised starts x_0 = s / ||s|| in FP32 (reading R7), rows padded to SST floats, components in the
+  // kernels' state slot order (xslot)
   constexpr int SST = round4(N);
   for (int s = blockIdx.x * blockDim.x + threadIdx.x; s < n_starts; s += gridDim.x * blockDim.x) {
     float v[N];
@@ -105,7 +146,10 @@ sshopm_pack_kernel(long long n_tensors, const float* __restrict__ entries, float
     for (int j = 0; j < N; ++j) { v[j] = starts[(size_t)s * N + j]; nn = fmaf(v[j], v[j], nn); }
     const float r = nn > 0.f ? rsqrtf(nn) : 0.f;
 #pragma unroll
-    for (int j = 0; j < SST; ++j) starts_n[(size_t)s * SST + j] = (j < N) ? v[j] * r : 0.f;
+    for (int j = 0; j < SST; ++j) starts_n[(size_t)s * SST + j] = 0.f;
+#pragma unroll
+    for (int j = 0; j < N; ++j) starts_n[(size_t)s * SST + xslot<M, N>(j)] = v[j] * r;   // state slot order
+    if constexpr (X21<M, N>::v) starts_n[(size_t)s * SST + 3] = v[1] * r;                 // (x2, x1) pair
   }
   // one tensor: coefficient-folded words w from its entries a, and its shift (alpha modes 1-3)
   auto row = [&](long long t, const float (&a)[S::U], float (&w)[S::PW]) {
@@ -201,6 +245,10 @@ struct Coefs {
   __device__ __forceinline__ void load(const float4* __restrict__ src) {
 #pragma unroll
     for (int i = 0; i < S::PW / 4; ++i) w[i] = ldg4(src + i);
+  }
+  __device__ __forceinline__ void load_if(bool p, const float4* __restrict__ src) {
+#pragma unroll
+    for (int i = 0; i < S::PW / 4; ++i) pld4(p, src + i, w[i]);
   }
   template <int I>
   __device__ __forceinline__ float word() const {
@@ -300,10 +348,16 @@ struct Coefs {
   }
 };
 
-// x stored in float2 slots: x_i = xs[i/2].x or .y
-template <int N>
+// State layout.  The N components of x live in the float2 slots xs[NX]:
+// generic shapes keep x_i in slot i (xs[i/2].x / .y); (4,3) keeps (x0, x2) in
+// xs[0] and x1 in xs[1].x ("X02"), so its degree-2/3 monomials are 7 FMUL2 +
+// 2 FMUL with no layout moves and the update is one FMUL2 + one FMUL
+// (tools/sassmodel: 75 instead of 88 modeled cycles per step on B200).  The
+// pack kernel writes the normalised starts in this slot order.
+template <int M, int N>
 __device__ __forceinline__ float xget(const float2 (&xs)[(N + 1) / 2], int i) {
-  return (i & 1) ? xs[i >> 1].y : xs[i >> 1].x;
+  const int s = xslot<M, N>(i);
+  return (s & 1) ? xs[s >> 1].y : xs[s >> 1].x;
 }
 
 // degree-(M-1) monomials x^q (lower list up to degree H, then left * right)
@@ -314,8 +368,8 @@ __device__ __forceinline__ void monomials(const float2 (&xs)[(N + 1) / 2], float
   static_for<S::NL>([&](auto tt) {
     constexpr int t = decltype(tt)::value;
     constexpr int par = S::T.low_parent[t], var = S::T.low_var[t];
-    if constexpr (par < 0) low[t] = xget<N>(xs, var);
-    else low[t] = low[par] * xget<N>(xs, var);
+    if constexpr (par < 0) low[t] = xget<M, N>(xs, var);
+    else low[t] = low[par] * xget<M, N>(xs, var);
   });
   static_for<S::Q>([&](auto qq) {
     constexpr int q = decltype(qq)::value;
@@ -325,13 +379,37 @@ __device__ __forceinline__ void monomials(const float2 (&xs)[(N + 1) / 2], float
   });
 }
 
-// (4,3): the paper's hand-unrolled case (Sec. V-D), paired for FFMA2/FMUL2.
-// x is held as (x0, x1), (x2, x1) so every degree-2 and degree-3 monomial pair
-// is one FMUL2 (8 instead of 16 FMUL); order = lex order of Tables<4,3>.
-template <int M, int N>
-struct X21 { static constexpr bool v = (M == 4 && N == 3); };
+// (4,3): the paper's hand-unrolled case (Sec. V-D).  With x in the X02
+// layout the ten degree-3 monomials (lex order q = 000 001 002 011 012 022 111
+// 112 122 222) come from 7 FMUL2 + 2 FMUL; Eq. 6 is scalar FFMA, q outer / j
+// inner (the monomial is the operand the three outputs share, so it is read
+// once); lambda = x . g as a scalar FMA chain (Definition 2).
+__device__ __forceinline__ float eval43(const Coefs<4, 3>& cf, const float2 (&xs)[2], float& g0, float& g1, float& g2) {
+  const float2 xq = xs[0];                    // (x0, x2)
+  const float x0 = xq.x, x2 = xq.y, x1 = xs[1].x;
+  const float2 a = __fmul2_rn(bc(x0), xq);    // x0x0, x0x2
+  const float2 b = __fmul2_rn(bc(x1), xq);    // x0x1, x1x2
+  const float2 c = f2(x1 * x1, x2 * x2);      // x1x1, x2x2
+  const float2 m0 = __fmul2_rn(bc(x0), a);    // q0 = 000, q2 = 002
+  const float2 m1 = __fmul2_rn(bc(x1), a);    // q1 = 001, q4 = 012
+  const float2 m2 = __fmul2_rn(bc(x1), b);    // q3 = 011, q7 = 112
+  const float2 m3 = __fmul2_rn(bc(c.y), xq);  // q5 = 022, q9 = 222
+  const float2 m4 = __fmul2_rn(bc(x1), c);    // q6 = 111, q8 = 122
+  const float mq[10] = {m0.x, m1.x, m0.y, m2.x, m1.y, m3.x, m4.x, m2.y, m4.y, m3.y};
+  // B-form words: (B_{q,0}, B_{q,1}) at 2q, B_{q,2} at 20 + q (Shape<4,3>: NP = 1, base = Q * NP * 2)
+  g0 = cf.template word<0>() * mq[0];
+  g1 = cf.template word<1>() * mq[0];
+  g2 = cf.template word<20>() * mq[0];
+  static_for<9>([&](auto qq) {
+    constexpr int q = decltype(qq)::value + 1;
+    g0 = fmaf(cf.template word<2 * q>(), mq[q], g0);
+    g1 = fmaf(cf.template word<2 * q + 1>(), mq[q], g1);
+    g2 = fmaf(cf.template word<20 + q>(), mq[q], g2);
+  });
+  return fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
+}
 
-#ifndef SSHOPM_SCALAR_MONO
+#if SSHOPM_43_FORM == 2 && !defined(SSHOPM_SCALAR_MONO)
 template <>
 __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
   const float2 x01 = xs[0], x21 = xs[1];
@@ -348,6 +426,31 @@ __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&m
   mq[5] = m45.y; mq[6] = m67.x; mq[7] = m67.y; mq[8] = m89.x; mq[9] = m89.y;
 }
 #endif
+
+// (4,3), natural layout (x0, x1 | x2): monomials from 7 FMUL2 + 2 FMUL; Eq. 6 as (g0, g1) FFMA2 with the
+// monomial broadcast plus g2 scalar FFMA on the same monomial (q outer).
+__device__ __forceinline__ float eval43n(const Coefs<4, 3>& cf, const float2 (&xs)[2], float2& g01, float& g2) {
+  const float2 x01 = xs[0];
+  const float x0 = x01.x, x1 = x01.y, x2 = xs[1].x;
+  const float2 a = __fmul2_rn(bc(x0), x01);   // x0x0, x0x1
+  const float2 b = __fmul2_rn(bc(x2), x01);   // x0x2, x1x2
+  const float2 c = f2(x1 * x1, x2 * x2);      // x1x1, x2x2
+  const float2 m0 = __fmul2_rn(bc(x0), a);    // q0 = 000, q1 = 001
+  const float2 m1 = __fmul2_rn(bc(x2), a);    // q2 = 002, q4 = 012
+  const float2 m2 = __fmul2_rn(bc(c.x), x01); // q3 = 011, q6 = 111
+  const float2 m3 = __fmul2_rn(bc(x2), b);    // q5 = 022, q8 = 122
+  const float2 m4 = __fmul2_rn(bc(x2), c);    // q7 = 112, q9 = 222
+  const float mq[10] = {m0.x, m0.y, m1.x, m2.x, m1.y, m3.x, m2.y, m4.x, m3.y, m4.y};
+  g2 = cf.template word<20>() * mq[0];
+  g01 = __fmul2_rn(cf.template pair<0>(), bc(mq[0]));
+  static_for<9>([&](auto qq) {
+    constexpr int q = decltype(qq)::value + 1;
+    g2 = fmaf(cf.template word<20 + q>(), mq[q], g2);
+    g01 = __ffma2_rn(cf.template pair<2 * q>(), bc(mq[q]), g01);
+  });
+  const float2 t = __fmul2_rn(x01, g01);
+  return fmaf(x2, g2, t.x + t.y);
+}
 
 // g = A x^{M-1} (pairs gp, odd tail gs) and lambda = x . g
 template <int M, int N>
@@ -384,7 +487,54 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
                                             float& lamp, int& k, bool& conv, bool& stop, bool has, float alpha,
                                             float la, float ls, float tol, int maxit) {
   using S = Shape<M, N>;
-  constexpr bool XL = X21<M, N>::v;
+  if constexpr (X02<M, N>::v) {
+    float g0, g1, g2;
+    lam = eval43(cf, xs, g0, g1, g2);                         // g = A x_k^3, lam_k = x_k . g
+    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));  // R2 (NaN lamp -> false)
+    const float x0 = xs[0].x, x2 = xs[0].y, x1 = xs[1].x;
+    float h0, h1, h2;                                         // xhat = +-(g + alpha x)   (Fig. 1 lines 2-5, R5)
+    if constexpr (SHIFT == 0) { h0 = g0; h1 = g1; h2 = g2; }
+    else if constexpr (SHIFT == 1) { h0 = fmaf(alpha, x0, g0); h1 = fmaf(alpha, x1, g1); h2 = fmaf(alpha, x2, g2); }
+    else if constexpr (SHIFT == 2) { h0 = fmaf(alpha, x0, -g0); h1 = fmaf(alpha, x1, -g1); h2 = fmaf(alpha, x2, -g2); }
+    else { h0 = fmaf(la, x0, g0 * ls); h1 = fmaf(la, x1, g1 * ls); h2 = fmaf(la, x2, g2 * ls); }
+    const float nn = fmaf(h2, h2, fmaf(h1, h1, h0 * h0));
+    const bool deg = !(nn >= 1.17549435e-38f);                  // R6 (FP32: subnormal counts as zero)
+    if constexpr (KIDLE) stop = conv | (k >= maxit) | deg;
+    else stop = (!has) | conv | (k >= maxit) | deg;
+    const float r = rsqrt_ftz(nn);                              // line 7: x = xhat / ||xhat||
+    if (!stop) {
+      xs[0] = __fmul2_rn(f2(h0, h2), bc(r));
+      xs[1].x = h1 * r;
+      lamp = lam;
+      ++k;
+    }
+    return;
+  } else if constexpr (N43<M, N>::v) {
+    float2 g01;
+    float g2;
+    lam = eval43n(cf, xs, g01, g2);
+    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
+    float2 h01;
+    float h2;
+    const float x2 = xs[1].x;
+    if constexpr (SHIFT == 0) { h01 = g01; h2 = g2; }
+    else if constexpr (SHIFT == 1) { h01 = __ffma2_rn(bc(alpha), xs[0], g01); h2 = fmaf(alpha, x2, g2); }
+    else if constexpr (SHIFT == 2) { h01 = __ffma2_rn(bc(alpha), xs[0], f2(-g01.x, -g01.y)); h2 = fmaf(alpha, x2, -g2); }
+    else { h01 = __ffma2_rn(bc(la), xs[0], __fmul2_rn(g01, bc(ls))); h2 = fmaf(la, x2, g2 * ls); }
+    const float2 u = __fmul2_rn(h01, h01);
+    const float nn = fmaf(h2, h2, u.x + u.y);
+    const bool deg = !(nn >= 1.17549435e-38f);
+    if constexpr (KIDLE) stop = conv | (k >= maxit) | deg;
+    else stop = (!has) | conv | (k >= maxit) | deg;
+    const float r = rsqrt_ftz(nn);
+    if (!stop) {
+      xs[0] = __fmul2_rn(h01, bc(r));
+      xs[1].x = h2 * r;
+      lamp = lam;
+      ++k;
+    }
+    return;
+  } else {
   float2 gp[S::NP > 0 ? S::NP : 1];
   float gs = 0.f;
   lam = evaluate<M, N>(cf, xs, gp, gs);                       // g = A x_k^{m-1}, lam_k = x_k . g
@@ -424,7 +574,7 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
   // FMUL2 / FMUL / MOV / IADD: no select per component (+9% step throughput
   // on B200, tools/microbench/step_loop.cu)
   if (!stop) {
-    if constexpr (XL) {
+    if constexpr (X21<M, N>::v) {
       xs[0] = __fmul2_rn(hp[0], bc(r));
       xs[1] = f2(hp[1].x * r, xs[0].y);
     } else {
@@ -434,6 +584,7 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
     }
     lamp = lam;
     ++k;
+  }
   }
 }
 
@@ -489,7 +640,6 @@ sshopm_solve_kernel(const SolveParams p) {
   using S = Shape<M, N>;
   using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
   constexpr int SST4 = round4(N) / 4;
-  constexpr bool XL = X21<M, N>::v;
 
   const int lane = threadIdx.x & 31;
   const uint32_t ltmask = lanemask_lt();
@@ -570,7 +720,7 @@ sshopm_solve_kernel(const SolveParams p) {
         p.out_lambda[item] = lam;
         float* ox = p.out_x + (size_t)item * N;              // one 64-bit row address, immediate offsets
 #pragma unroll
-        for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
+        for (int j = 0; j < N; ++j) ox[j] = xget<M, N>(xs, j);
         p.out_iters[item] = k;
         p.out_conv[item] = conv ? 1 : 0;
       }
@@ -615,8 +765,7 @@ sshopm_solve_kernel(const SolveParams p) {
           v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
         }
 #pragma unroll
-        for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
-        if constexpr (XL) xs[1].y = v[1];                  // (x2, x1) layout
+        for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);   // starts_n is in slot order
       }
       k = ok ? 0 : (stop ? 0x7fffffff : k);                  // idle lanes: k >= maxit keeps them stopped
       lamp = ok ? __int_as_float(0x7fffffff) : lamp;         // NaN: the first test never fires (reading R2)
@@ -682,6 +831,134 @@ sshopm_solve_kernel(const SolveParams p) {
 }
 
 
+// ------------------------------------------------- solve kernel, schedule 6 --
+// Item per lane with a branch-free refill (opt-in; measured 1.5% slower than schedule 1 at C2 with the
+// same step, profiles/r2/solve_variants.md).  Each warp owns one chunk of
+// consecutive items [c_next, c_end) at a time (items are tensor-major: item =
+// t * S + s) and claims the next chunk from the global counter only when the
+// current one is used up; the claim for the following chunk is issued one
+// chunk ahead, so the atomic's latency is off the critical path.  A refill
+// (once >= K lanes are stopped at a trip boundary) is straight-line predicated
+// code: stores of the stopped lanes' results, rank = popc of the stopped
+// lanes below, item = c_next + rank, one LDG.128 row load per 4 coefficient
+// words and one start load.  Lanes beyond the chunk's remaining items go idle
+// (k = IDLE) until the next refill.  Results are bitwise those of the other
+// schedules (same per-step arithmetic, sshopm_step).
+template <int M, int N, int SHIFT, bool WIDE>
+__global__ void __launch_bounds__(256, Shape<M, N>::MINB)
+sshopm_solve_lean_kernel(const SolveParams p) {
+  constexpr int STEPS = steps_per_trip<M, N>();
+  using S = Shape<M, N>;
+  using Idx = typename std::conditional<WIDE, unsigned long long, uint32_t>::type;
+  constexpr int SST4 = round4(N) / 4;
+  constexpr int IDLE = 0x7fffffff;                       // k of a lane without an item (>= any maxit)
+
+  const int lane = threadIdx.x & 31;
+  const uint32_t ltmask = lanemask_lt();
+  const uint32_t FULL = 0xffffffffu;
+  const float alpha = (SHIFT == 2) ? -p.alpha : p.alpha;
+  const float tol = p.tol;
+  const int maxit = p.maxit;
+  const uint32_t S_ = (uint32_t)p.S;
+  const Idx total = (Idx)p.n_tensors * (Idx)S_;
+  const Idx chunk_items = (Idx)p.chunk_tensors * (Idx)S_;
+  const unsigned int n_chunks = (unsigned int)p.n_chunks;
+
+  Idx c_next = 0, c_end = 0;                             // warp-uniform current chunk
+  unsigned int pref = 0;                                 // next chunk index (claimed one chunk ahead)
+  if (lane == 0) pref = atom_add1(p.counter);
+  bool exhausted = false;
+  uint32_t k_eff = (uint32_t)p.refill_k;
+
+  Coefs<M, N> cf;
+  float2 xs[S::NX];
+#pragma unroll
+  for (int i = 0; i < S::NX; ++i) xs[i] = f2(0.f, 0.f);
+  float lamp = 0.f, lam = 0.f;
+  int k = IDLE;
+  bool stop = true, conv = false;
+  Idx item = 0;
+  float la = 0.f, ls = 1.f;
+  uint32_t it_sum = 0;
+
+  for (;;) {
+    const uint32_t smask = __ballot_sync(FULL, stop);
+    const uint32_t cnt = __popc(smask);
+    if (cnt >= k_eff) {
+      if (c_next == c_end && !exhausted) {               // warp-uniform: take the prefetched chunk, prefetch the next
+        const unsigned int ch = __shfl_sync(FULL, pref, 0);
+        if (ch < n_chunks) {
+          c_next = (Idx)ch * chunk_items;
+          c_end = c_next + chunk_items < total ? c_next + chunk_items : total;
+          if (lane == 0) pref = atom_add1(p.counter);
+        } else {
+          exhausted = true;
+          k_eff = 32u;
+        }
+      }
+      // results of the lanes that stopped (A7): predicated stores
+      const bool wr = stop && (k != IDLE);
+      pst(wr, p.out_lambda + item, lam);
+#pragma unroll
+      for (int j = 0; j < N; ++j) pst(wr, p.out_x + (size_t)item * N + j, xget<M, N>(xs, j));
+      pst(wr, p.out_iters + item, (int32_t)k);
+      pst(wr, p.out_conv + item, conv ? 1u : 0u);
+      it_sum += wr ? (uint32_t)k : 0u;
+      // next items: rank among the stopped lanes, within the chunk's remaining items
+      const uint32_t rank = __popc(smask & ltmask);
+      const Idx avail = c_end - c_next;
+      const bool ok = stop && (Idx)rank < avail;
+      item = ok ? c_next + (Idx)rank : item;
+      Idx tv;
+      uint32_t s;
+      if (p.s_log2 >= 0) {                               // S a power of two (the paper's 128): shift and mask
+        tv = item >> p.s_log2;
+        s = (uint32_t)item & (S_ - 1u);
+      } else if constexpr (WIDE) {
+        tv = item / S_;
+        s = (uint32_t)(item - tv * S_);
+      } else {
+        tv = fast_div(item, p.divS);
+        s = item - tv * S_;
+      }
+      if constexpr (SHIFT == 3) {
+        float at = 0.f;
+        if (ok) at = __ldg(p.alpha_t + tv);
+        ls = ok ? (at >= 0.f ? 1.f : -1.f) : ls;         // Fig. 1 lines 2-5 (R5: alpha = 0 -> "+")
+        la = ok ? fabsf(at) : la;
+      }
+      cf.load_if(ok, p.packed + tv * (Idx)(S::PW / 4));
+      {
+        float4 v[SST4];
+#pragma unroll
+        for (int i = 0; i < SST4; ++i) {
+          v[i] = make_float4(xs[2 * i].x, xs[2 * i].y, (2 * i + 1 < S::NX) ? xs[2 * i + 1].x : 0.f,
+                             (2 * i + 1 < S::NX) ? xs[2 * i + 1].y : 0.f);
+          pld4(ok, p.starts_n + s * SST4 + i, v[i]);     // starts_n is in slot order
+        }
+#pragma unroll
+        for (int i = 0; i < S::NX; ++i)
+          xs[i] = (i % 2 == 0) ? f2(v[i / 2].x, v[i / 2].y) : f2(v[i / 2].z, v[i / 2].w);
+      }
+      lamp = ok ? __int_as_float(0x7fffffff) : lamp;     // NaN: the first test never fires (reading R2)
+      k = stop ? (ok ? 0 : IDLE) : k;
+      c_next += (Idx)cnt < avail ? (Idx)cnt : avail;
+      if (exhausted && __ballot_sync(FULL, k != IDLE) == 0u) break;
+    }
+#pragma unroll
+    for (int rep = 0; rep < STEPS; ++rep)
+      sshopm_step<M, N, SHIFT, true>(cf, xs, lam, lamp, k, conv, stop, true, alpha, la, ls, tol, maxit);
+  }
+
+  if (p.total_iters) {
+    unsigned long long ws = it_sum;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(0xffffffffu, ws, o);
+    if (lane == 0) atomicAdd(p.total_iters, ws);
+  }
+}
+
+
 // ------------------------------------------- solve kernel, tensor-per-lane --
 // Schedule 2: a lane owns one tensor at a time and
 // walks its S starts in order, so its coefficient registers are loaded once
@@ -696,7 +973,6 @@ sshopm_solve_tpl_kernel(const SolveParams p) {
   using S = Shape<M, N>;
   using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
   constexpr int SST4 = round4(N) / 4;
-  constexpr bool XL = X21<M, N>::v;
 
   const int lane = threadIdx.x & 31;
   const uint32_t ltmask = lanemask_lt();
@@ -729,7 +1005,7 @@ sshopm_solve_tpl_kernel(const SolveParams p) {
           p.out_lambda[item] = lam;
           float* ox = p.out_x + (size_t)item * N;
 #pragma unroll
-          for (int j = 0; j < N; ++j) ox[j] = xget<N>(xs, j);
+          for (int j = 0; j < N; ++j) ox[j] = xget<M, N>(xs, j);
           p.out_iters[item] = k;
           p.out_conv[item] = conv ? 1 : 0;
           it_sum += (unsigned long long)k;
@@ -763,8 +1039,7 @@ sshopm_solve_tpl_kernel(const SolveParams p) {
           v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
         }
 #pragma unroll
-        for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
-        if constexpr (XL) xs[1].y = v[1];
+        for (int i = 0; i < S::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);   // starts_n is in slot order
         k = 0;
         lamp = __int_as_float(0x7fffffff);
       }
@@ -942,18 +1217,39 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
     cf.load(packed + i * (S::PW / 4));
     float2 xs[S::NX];
 #pragma unroll
-    for (int t = 0; t < S::NX; ++t)
-      xs[t] = f2(__ldg(x + i * N + 2 * t), (2 * t + 1 < N) ? __ldg(x + i * N + 2 * t + 1) : 0.f);
+    for (int t = 0; t < S::NX; ++t) xs[t] = f2(0.f, 0.f);
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const int sl = xslot<M, N>(j);
+      if (sl & 1) xs[sl >> 1].y = __ldg(x + i * N + j);
+      else xs[sl >> 1].x = __ldg(x + i * N + j);
+    }
     if constexpr (X21<M, N>::v) xs[1].y = xs[0].y;
-    float2 gp[S::NP > 0 ? S::NP : 1];
-    float gs = 0.f;
-    const float lam = evaluate<M, N>(cf, xs, gp, gs);
-    static_for<S::NP>([&](auto pp) {
-      constexpr int q = decltype(pp)::value;
-      out_g[i * N + 2 * q] = gp[q].x;
-      out_g[i * N + 2 * q + 1] = gp[q].y;
-    });
-    if constexpr (S::ODD) out_g[i * N + N - 1] = gs;
+    float lam;
+    if constexpr (N43<M, N>::v) {
+      float2 g01;
+      float g2;
+      lam = eval43n(cf, xs, g01, g2);
+      out_g[i * N + 0] = g01.x;
+      out_g[i * N + 1] = g01.y;
+      out_g[i * N + 2] = g2;
+    } else if constexpr (X02<M, N>::v) {
+      float g0, g1, g2;
+      lam = eval43(cf, xs, g0, g1, g2);
+      out_g[i * N + 0] = g0;
+      out_g[i * N + 1] = g1;
+      out_g[i * N + 2] = g2;
+    } else {
+      float2 gp[S::NP > 0 ? S::NP : 1];
+      float gs = 0.f;
+      lam = evaluate<M, N>(cf, xs, gp, gs);
+      static_for<S::NP>([&](auto pp) {
+        constexpr int q = decltype(pp)::value;
+        out_g[i * N + 2 * q] = gp[q].x;
+        out_g[i * N + 2 * q + 1] = gp[q].y;
+      });
+      if constexpr (S::ODD) out_g[i * N + N - 1] = gs;
+    }
     out_lam[i] = lam;
   }
 }

@@ -32,6 +32,9 @@ P3 Eigenvector angle <= 1e-3 rad between x_gpu and the oracle iterate at the
 P4 Fixed-K (tol < 0): |lam_gpu - lam_ref| <= max(1e-5 max(1,|lam|), 1e3 s), s =
    max oracle lambda_K change over the witnesses.
 """
+import json
+import os
+
 import numpy as np
 
 from oracle import sshopm as O
@@ -252,3 +255,16 @@ def fixed_k_parity(ent, starts, m, n, alpha, K, lam_g):
             s = np.maximum(s, np.abs(wl.astype(np.float64) - lam_r[vox, st]))
         unexpl = int(np.sum(d[vox, st] > np.maximum(FIXED_TOL * scale[vox, st], 1e3 * s)))
     return {"max_rel": float((d / scale).max()), "outliers": int(len(bad)), "unexplained": unexpl}
+
+
+def record(name, rep):
+    """Save a parity report as JSON under <repo>/gpurun_out/parity/ (best effort; never fails a test)."""
+    try:
+        root = os.environ.get("GRAFT_REPO_ROOT") or os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+        d = os.path.join(root, "gpurun_out", "parity")
+        os.makedirs(d, exist_ok=True)
+        safe = "".join(c if c.isalnum() or c in "-_.[]," else "_" for c in name)
+        with open(os.path.join(d, safe + ".json"), "w") as f:
+            json.dump(rep, f, default=lambda o: o.item() if hasattr(o, "item") else str(o))
+    except OSError:
+        pass

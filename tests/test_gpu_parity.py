@@ -30,9 +30,26 @@ def _solve(dev, m, n, ent, st, alpha, tol, maxit, **kw):
     return tuple(t.cpu().numpy() for t in out)
 
 
+_CURRENT = {"name": None}
+
+
+@pytest.fixture(autouse=True)
+def _test_name(request):
+    _CURRENT["name"] = request.node.name
+    yield
+    _CURRENT["name"] = None
+
+
+def _record(rep, **extra):
+    """Write the parity report of the running test to gpurun_out/parity/<test>.json (the auditable evidence
+    of how many lanes each rule explained; summarised under profiles/ by tools/parity_summary.py)."""
+    PR.record(_CURRENT["name"] or "unnamed", dict(rep, **extra))
+
+
 def _assert_parity(rep, max_sensitive=1e-3):
     """P1-P3 with zero unexplained lanes; explained (precision-sensitive) lanes must stay rare."""
     print({k: v for k, v in rep.items() if k != "details"})
+    _record(rep, max_sensitive=max_sensitive)
     assert rep["flag_unexplained"] == 0, rep
     assert rep["lam_unexplained"] == 0, rep
     assert rep.get("angle_unexplained", 0) == 0, rep
@@ -107,6 +124,25 @@ def test_fixed_k(dev, alpha, K):
     assert (it == K).all() and not cv.any()
     r = PR.fixed_k_parity(ent, st, m, n, alpha, K, lam)
     print(r)
+    _record(r)
+    assert r["unexplained"] == 0, r
+
+
+@pytest.mark.parametrize("K", [1, 5, 10])
+@pytest.mark.parametrize("m,n,V,alpha,schedule", [(6, 3, 96, 0.25, 0), (8, 3, 24, 0.5, 0), (4, 6, 48, 0.0, 0),
+                                                  (4, 3, 64, 0.5, 5), (5, 4, 24, 4.0, 5), (6, 4, 16, 0.5, 3),
+                                                  (4, 3, 64, 0.0, 2)])
+def test_fixed_k_shapes(dev, m, n, V, alpha, schedule, K):
+    """Fixed-K lambda (tol < 0: exactly K updates, Fig. 1) within 1e-5 relative of the FP64 oracle (P4) for
+    the C3 / C4a / C4b shapes on their unrolled kernels, the blocked (5) and item-per-lane (3) table-driven
+    kernels and the tensor-per-lane schedule (2)."""
+    ent = syn.gen_voxels(m, n, 300, V, 6) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 6)
+    st = syn.gen_starts(64, n, 3)
+    lam, x, it, cv = _solve(dev, m, n, ent, st, alpha, -1.0, K, schedule=schedule)
+    assert (it == K).all() and not cv.any()
+    r = PR.fixed_k_parity(ent, st, m, n, alpha, K, lam)
+    print(r)
+    _record(r)
     assert r["unexplained"] == 0, r
 
 
@@ -144,7 +180,9 @@ def test_invariance_across_launch_configs(dev):
     base = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
     for kw in [dict(refill_threshold=1), dict(refill_threshold=32), dict(ctas_per_sm=1),
                dict(refill_threshold=5, ctas_per_sm=2), {}, dict(schedule=2), dict(schedule=2, refill_threshold=3),
-               dict(schedule=2, ctas_per_sm=1, refill_threshold=32), dict(schedule=1)]:
+               dict(schedule=2, ctas_per_sm=1, refill_threshold=32), dict(schedule=1), dict(schedule=6),
+               dict(schedule=6, refill_threshold=3), dict(schedule=1, chunk_tensors=1),
+               dict(schedule=1, chunk_tensors=7, refill_threshold=2)]:
         other = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100, **kw)
         for a, b in zip(base, other):
             assert np.array_equal(a, b), kw
@@ -195,6 +233,19 @@ def test_dedup_end_to_end_vs_oracle(dev):
     assert np.array_equal(mu[same], om[same])
     filled = rp[same] >= 0
     assert np.all(np.abs(cl[same][filled] - ol[same][filled]) <= 1e-4 * np.maximum(1, np.abs(ol[same][filled])))
+    # representatives' eigenvectors: angle to the oracle iterate of the same lane at the GPU's own
+    # iteration count (trajectory alignment, parity rule P3), sign-free for even m
+    vox, slot = np.nonzero(rp >= 0)
+    keep = same[vox]
+    vox, slot = vox[keep], slot[keep]
+    st_i = rp[vox, slot]
+    k_gpu = it.cpu().numpy()[vox, st_i]
+    full = O.expand_full(ent, m, n)
+    _, xk, _, _ = O.sshopm_lanes(lambda idx: full[vox[idx]], O.normalise_starts(st)[st_i], 0.0, -1.0,
+                                 int(k_gpu.max()), k_gpu)
+    ang = PR.angle(cx[vox, slot], xk, True)
+    _record({"representatives": int(len(vox)), "angle_max": float(ang.max()), "voxels_compared": int(same.sum())})
+    assert ang.max() <= PR.ANG_TOL, ang.max()
 
 
 @pytest.mark.parametrize("S", [16, 100, 128, 200])
@@ -242,7 +293,7 @@ def test_run_host_matches_device_path(dev):
     assert out["total_iters"] == int(it.cpu().numpy().sum())
 
 
-@pytest.mark.parametrize("schedule", [1, 2])
+@pytest.mark.parametrize("schedule", [1, 2, 6])
 @pytest.mark.parametrize("V,S", [(1, 1), (3, 1), (5, 7), (40, 2), (2, 300)])
 def test_tiny_chunks(dev, V, S, schedule):
     """Chunks smaller than a warp's request (S * tensors < 32) must not overrun (regression)."""
@@ -295,6 +346,41 @@ def test_fused_equals_two_pass(dev, m, n, V, S, alpha, kmax):
     rb, db = _fused(dev, m, n, ent, st, alpha, 1e-6, 100, 1e-2, 0.05, kmax)
     for a, b in zip(ra + da, rb + db):
         assert np.array_equal(a, b)
+
+
+def test_fused_vs_oracle(dev):
+    """The fused solve->dedup path against the FP64 oracle directly: its per-start outputs pass the parity
+    contract (P1-P3) and its records equal the oracle's R16 rule applied to the same lanes; on voxels without
+    a flag difference, cluster counts / representatives / multiplicities equal oracle solve + oracle dedup."""
+    m, n, V, S = 4, 3, 600, 128
+    ent = syn.gen_voxels(m, n, 2000, V, 7)
+    st = syn.gen_starts(S, n, 0)
+    raw, dd = _fused(dev, m, n, ent, st, 0.0, 1e-6, 100, 1e-2, 0.05, 8)
+    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, tuple(raw)))
+    oc, ol, ox, om, orp = D.dedup(raw[0], raw[1], raw[3].astype(bool), m, 1e-2, 0.05, 8)
+    for a, b in zip(dd, (oc, ol, ox, om, orp)):
+        assert np.array_equal(np.asarray(a).astype(np.float64), np.asarray(b).astype(np.float64))
+    rl, rx, ri, rc = O.sshopm(ent, st, m, n, 0.0, 1e-6, 100)
+    oc2, ol2, ox2, om2, orp2 = D.dedup(rl, rx, rc, m, 1e-2, 0.05, 8)
+    same = ~np.any(raw[3].astype(bool) != rc, axis=1)
+    assert same.mean() > 0.98
+    assert np.array_equal(dd[0][same], oc2[same]) and np.array_equal(dd[4][same], orp2[same])
+    assert np.array_equal(dd[3][same], om2[same])
+
+
+def test_plain_sshopm_solve_entry_point(dev):
+    """sshopm_solve itself: library defaults and its own cudaMallocAsync workspace, data on
+    the GPU; bitwise equal to sshopm_solve_ex and within the parity contract."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 100, 512, 2)
+    st = syn.gen_starts(128, n, 1)
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    a = [u.cpu().numpy() for u in s.solve_plain(e, t, 0.0, 1e-6, 100)]
+    b = [u.cpu().numpy() for u in s.solve(e, t, 0.0, 1e-6, 100)]
+    for u, v in zip(a, b):
+        assert np.array_equal(u, v)
+    _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, tuple(a)))
 
 
 def test_fused_ring_overflow(dev):
@@ -384,7 +470,9 @@ def test_general_solve_parity(dev, m, n, V, alpha, schedule):
     ent = syn.gen_voxels(m, n, 0, V, 3) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 3)
     st = syn.gen_starts(64, n, 1)
     gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 200, schedule=schedule)
-    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 200, gpu), 0.05)
+    # even m with alpha >= 0 (structured voxel tensors): the benchmark bar, <= 0.1% precision-sensitive lanes;
+    # odd m (unstructured tensors, sign-flip trajectories) keeps the stress bar
+    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 200, gpu), 1e-3 if m % 2 == 0 else 0.05)
 
 
 @pytest.mark.parametrize("shift", ["auto_max", "auto_min"])
@@ -416,7 +504,7 @@ def test_blocked_solve_parity(dev, m, n, V, S, alpha):
     ent = syn.gen_voxels(m, n, 0, V, 5) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 5)
     st = syn.gen_starts(S, n, 4)
     gpu = _solve(dev, m, n, ent, st, alpha, 1e-6, 300, schedule=5)
-    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 300, gpu), 0.05)
+    _assert_parity(PR.solve_parity(ent, st, m, n, alpha, 1e-6, 300, gpu), 1e-3 if m % 2 == 0 else 0.05)
 
 
 @pytest.mark.parametrize("shift", ["auto_max", "auto_min", "per_tensor"])

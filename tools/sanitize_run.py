@@ -1,0 +1,52 @@
+"""Small runs of every solve / dedup path for compute-sanitizer (memcheck, racecheck, synccheck, initcheck):
+    compute-sanitizer --tool racecheck python tools/sanitize_run.py <case>
+cases: two_pass (C1 tensors x 128 starts, default schedule: pack + lean solve + dedup), legacy (schedule 6),
+tpl (schedule 2), fused (fuse_dedup = 1: in-kernel ring + list kernel, forced overflow), blocked ((4,10),
+V = 6, schedule 5, two tensor buffers per warp), general (schedule 3), classify, run_host."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+import synthetic as syn  # noqa: E402
+import paper_conf_ipps_ballardkp11_b200 as sh  # noqa: E402
+
+case = sys.argv[1] if len(sys.argv) > 1 else "two_pass"
+dev = torch.device("cuda:0")
+
+
+def t(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+
+
+if case in ("two_pass", "legacy", "tpl", "fused", "classify"):
+    V = 1024 if case != "fused" else 2000
+    ent = syn.gen_voxels(4, 3, 0, V, 0)
+    if case == "fused":
+        ent[::40] = syn.gen_uniform_tensors(4, 3, V // 40, 9)   # slow lanes: ring overflow
+    st = syn.gen_starts(128, 3, 0)
+    s = sh.Solver(4, 3)
+    if case == "fused":
+        s.solve_dedup(t(ent), t(st), 0.0, 1e-6, 1000, 1e-2, 0.05, 4, fused=True)
+    else:
+        sched = {"two_pass": 0, "legacy": 6, "tpl": 2, "classify": 0}[case]
+        lam, x, it, cv = s.solve(t(ent), t(st), 0.0, 1e-6, 100, schedule=sched)
+        cnt, cl, cx, mu, rp = s.dedup(lam, x, cv, 1e-2, 0.05, 8)
+        if case == "classify":
+            s.classify(t(ent), cnt, cl, cx, 1e-3)
+elif case == "blocked":
+    ent = syn.gen_voxels(4, 10, 0, 6, 5)
+    st = syn.gen_starts(32, 10, 4)
+    sh.Solver(4, 10).solve(t(ent), t(st), 0.0, 1e-6, 300, schedule=5)
+elif case == "general":
+    ent = syn.gen_voxels(6, 4, 0, 16, 3)
+    st = syn.gen_starts(64, 4, 1)
+    sh.Solver(6, 4).solve(t(ent), t(st), 0.5, 1e-6, 200, schedule=3)
+elif case == "run_host":
+    ent = syn.gen_voxels(4, 3, 0, 3000, 9)
+    st = syn.gen_starts(128, 3, 0)
+    sh.Solver(4, 3).run_host(ent, st, 0.0, 1e-6, 100, 1e-2, 0.05, 8, raw=True, chunk_tensors=700)
+torch.cuda.synchronize()
+print("ok", case)
