@@ -118,7 +118,7 @@ template <int M, int N>
 struct N43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 1); };
 // form 2: the round-1 layout, x held as (x0, x1), (x2, x1) (slot 3 duplicates x1), monomials as 8 FMUL2
 template <int M, int N>
-struct X21 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 2); };
+struct X21 { static constexpr bool v = (M == 4 && N == 3 && (SSHOPM_43_FORM == 2 || SSHOPM_43_FORM == 3)); };
 template <int M, int N>
 __host__ __device__ constexpr int xslot(int i) {
   return X02<M, N>::v ? (i == 0 ? 0 : (i == 1 ? 2 : 1)) : i;
@@ -424,6 +424,22 @@ __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&m
   const float2 m89 = __fmul2_rn(bc(s2.y), x12);   // 122 222
   mq[0] = m01.x; mq[1] = m01.y; mq[2] = m23.x; mq[3] = m23.y; mq[4] = m45.x;
   mq[5] = m45.y; mq[6] = m67.x; mq[7] = m67.y; mq[8] = m89.x; mq[9] = m89.y;
+}
+#elif SSHOPM_43_FORM == 3
+// form 3: the form-2 layout without the (x1, x2) pair (no register moves): every product pairs with (x2, x1)
+template <>
+__device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
+  const float2 x01 = xs[0], x21 = xs[1];
+  const float2 s0 = __fmul2_rn(bc(x01.x), x01);   // (x0x0, x0x1)
+  const float2 s1 = __fmul2_rn(x01, x21);         // (x0x2, x1x1)
+  const float2 s2 = __fmul2_rn(bc(x21.x), x21);   // (x2x2, x2x1)
+  const float2 m01 = __fmul2_rn(bc(x01.x), s0);   // 000 001
+  const float2 m23 = __fmul2_rn(bc(x01.x), s1);   // 002 011
+  const float2 m54 = __fmul2_rn(bc(x01.x), s2);   // 022 012
+  const float2 m76 = __fmul2_rn(bc(s1.y), x21);   // 112 111
+  const float2 m98 = __fmul2_rn(bc(s2.x), x21);   // 222 122
+  mq[0] = m01.x; mq[1] = m01.y; mq[2] = m23.x; mq[3] = m23.y; mq[4] = m54.y;
+  mq[5] = m54.x; mq[6] = m76.y; mq[7] = m76.x; mq[8] = m98.y; mq[9] = m98.x;
 }
 #endif
 
