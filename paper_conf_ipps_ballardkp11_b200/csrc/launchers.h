@@ -12,6 +12,7 @@ struct Launchers {
   int bform;                 // 1 if the B-form (coefficient-folded) registers are used
   int default_refill;
   int default_schedule;
+  int (*wt_smem_per_warp)(int S);       // schedule 7 staging bytes per warp
   void (*class_index)(int32_t* out);   // [U][m], 0-based
   cudaError_t (*occupancy)(int shift, bool wide, int schedule, int fused, int smem_bytes, int* blocks_per_sm);
   cudaError_t (*pack)(long long n_tensors, const float* entries, float4* packed, unsigned int* counter, int n_starts,

@@ -59,8 +59,8 @@ int chunk_tensors_for(int S) { return (S >= 256) ? 1 : (256 + S - 1) / S; }
 static size_t packed_region(const Launchers* L, int64_t N) { return ((size_t)N * (size_t)L->PW * 4 + 255) / 256 * 256; }
 
 static size_t chunk_list_region(int64_t N, int S) {
-  const size_t n_chunks = S > 0 ? (size_t)((N + chunk_tensors_for(S) - 1) / chunk_tensors_for(S)) : 0;
-  return (n_chunks * 4 + 255) / 256 * 256;
+  (void)S;   // one entry per tensor: chunk indices (schedule 1 fused ring) or tensor indices (schedule 7)
+  return ((size_t)N * 4 + 255) / 256 * 256;
 }
 
 size_t workspace_bytes(const Launchers* L, int64_t N, int S) {
@@ -273,7 +273,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const Launchers* L = h->L;
   const int sms = device_sms();
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve: no device");
-  if (opts && (opts->schedule < 0 || opts->schedule > 6)) return SSHOPM_EINVAL;
+  if (opts && (opts->schedule < 0 || opts->schedule > 7)) return SSHOPM_EINVAL;
   if (!L || (opts && opts->schedule >= 3 && opts->schedule <= 5)) {   // table-driven general kernel (any (m, n))
     if (!h->gen) return SSHOPM_EUNSUPPORTED;
     int rc = general_solve(h->gen, N, d_entries, S, d_starts, alpha, tol, maxit, d_out_lambda, d_out_x, d_out_iters,
@@ -300,10 +300,22 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   // schedule: 1 = item per lane (two-chunk refill, default), 2 = tensor per lane, 6 = item per lane with the
   // lean predicated refill (C2: 4.33 vs 4.26 ms for schedule 1, profiles/r2/solve_variants.md)
   int schedule = (opts && opts->schedule > 0) ? opts->schedule : L->default_schedule;
-  if (schedule != 1 && schedule != 2 && schedule != 6) return SSHOPM_EINVAL;   // 3-5 (general) handled above
+  if (schedule != 1 && schedule != 2 && schedule != 6 && schedule != 7) return SSHOPM_EINVAL;   // 3-5: general
   if (shift == 3 && schedule == 2) schedule = 1;                 // per-tensor alpha: not on schedule 2
+  // records-only request (opts->fuse_dedup = 2): the warp-tensor pipeline clusters in the solve kernel and
+  // writes per-start outputs only for tensors it cannot cluster in registers (> 32 clusters)
+  if (dd && opts && opts->fuse_dedup == 2) schedule = 7;
+  int wt_mode = 0, wt_smem = 0;
+  if (schedule == 7) {
+    const int per_warp = L->wt_smem_per_warp(S);
+    wt_mode = dd && opts && opts->fuse_dedup == 2 ? 1 : (dd && opts && opts->fuse_dedup == 1 ? 2 : 0);
+    if (wt_mode && S != 128) wt_mode = 0;                        // in-kernel clustering: S = 128 register form
+    wt_smem = 8 * per_warp;
+    if (wt_smem > 200 * 1024) { schedule = 1; wt_mode = 0; }     // staging does not fit: schedule 1
+  }
   int bps = 0;
-  cudaError_t e = cached_occupancy(h, shift, wide, schedule, &bps);
+  cudaError_t e = schedule == 7 ? L->occupancy(shift, false, 7, wt_mode, wt_smem, &bps)
+                                : cached_occupancy(h, shift, wide, schedule, &bps);
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_solve: occupancy");
   if (bps < 1) bps = 1;
   // fused dedup (opt-in, opts->fuse_dedup = 1): schedule 1, S <= 1024, and only if its shared memory
@@ -313,7 +325,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   int smem = 0;
   const bool fregs = dd && S == 128 && ((uintptr_t)d_out_lambda % 16 == 0) && ((uintptr_t)d_out_x % 16 == 0) &&
                      ((uintptr_t)d_out_converged % 4 == 0);
-  if (dd && schedule != 2 && S <= 1024 && opts && opts->fuse_dedup == 1) {
+  if (dd && (schedule == 1 || schedule == 6) && S <= 1024 && opts && opts->fuse_dedup == 1) {
     const int fs = 8 * fused_smem_words(S, L->n, fregs) * 4;
     int fb = 0;
     if (fs <= 200 * 1024 && L->occupancy(shift, wide, schedule, fregs ? 2 : 1, fs, &fb) == cudaSuccess && fb >= bps) {
@@ -338,7 +350,9 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   const long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
   if (n_chunks >= (1LL << 32) - (1LL << 20) || N >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
   long long grid = (long long)sms * bps;
-  if (schedule != 2) {
+  if (schedule == 7) {
+    if (grid * 8 > N) grid = (N + 7) / 8;                          // warps claim whole tensors
+  } else if (schedule != 2) {
     if (grid * 8 > n_chunks) grid = (n_chunks + 7) / 8;
   } else {
     if (grid * 256 > N) grid = (N + 255) / 256;
@@ -369,6 +383,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   p.S = S;
   p.divS = make_fastdiv((uint32_t)S);
   p.s_log2 = -1;
+  p.s_mask = (uint32_t)S - 1u;
   if ((S & (S - 1)) == 0)
     for (int b = 0; b < 31; ++b)
       if ((1 << b) == S) p.s_log2 = b;
@@ -385,11 +400,13 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   p.ovf_count = ws.ovf_count;
   p.ovf_list = ws.ovf_list;
   p.fused_regs = fregs ? 1 : 0;
-  e = L->solve(p, shift, wide, schedule, fused, (int)grid, smem, st);
+  if (schedule == 7) { fused = wt_mode; smem = wt_smem; }
+  e = L->solve(p, shift, schedule == 7 ? false : wide, schedule, fused, (int)grid, smem, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
   h->launches.fetch_add(2);
   if (dd) {
-    if (fused) rc = launch_dedup_list(h->m, h->n, p.dd, ws.ovf_count, ws.ovf_list, chunk_tensors, st);
+    if (schedule == 7 && wt_mode) rc = launch_dedup_list(h->m, h->n, p.dd, ws.ovf_count, ws.ovf_list, 1, st);
+    else if (fused) rc = launch_dedup_list(h->m, h->n, p.dd, ws.ovf_count, ws.ovf_list, chunk_tensors, st);
     else rc = launch_dedup(h->m, h->n, p.dd, st);
     if (rc != SSHOPM_OK) { release_workspace(&ws, st); return rc; }
     h->launches.fetch_add(1);

@@ -18,8 +18,19 @@ void class_index(int32_t* out) {
     for (int t = 0; t < M; ++t) out[c * M + t] = T.cls_idx[c][t];
 }
 
+template <int SH, int MODE>
+const void* wt_fn() { return reinterpret_cast<const void*>(sshopm_solve_wt_kernel<M, N, SH, MODE>); }
+
 template <int SH, bool W, int F>
 cudaError_t occ2(int schedule, int smem, int* bps) {
+  if (schedule == 7) {   // warp-tensor pipeline: F = MODE (0 raw, 1 records only, 2 both); smem = staging bytes
+    const void* fn = wt_fn<SH, F>();
+    if (smem > 48 * 1024) {
+      cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      if (e != cudaSuccess) return e;
+    }
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, fn, 256, smem);
+  }
   if constexpr (SH == 3) {
     if (schedule == 2) return cudaErrorInvalidValue;         // per-tensor alpha: schedule 1 only
   } else {
@@ -49,6 +60,18 @@ cudaError_t occupancy(int shift, bool wide, int schedule, int fused, int smem, i
 
 template <int SH, bool W, int F>
 cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaStream_t st) {
+  if (schedule == 7) {
+    if constexpr (!W) {
+      if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(sshopm_solve_wt_kernel<M, N, SH, F>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+      }
+      sshopm_solve_wt_kernel<M, N, SH, F><<<grid, 256, smem, st>>>(p);
+      return cudaGetLastError();
+    }
+    return cudaErrorInvalidValue;                            // the api launches schedule 7 with W = false
+  }
   if (schedule == 2) {
     if constexpr (SH == 3) return cudaErrorInvalidValue;     // per-tensor alpha: schedule 1 only
     else sshopm_solve_tpl_kernel<M, N, SH, W><<<grid, 256, 0, st>>>(p);
@@ -99,10 +122,12 @@ cudaError_t apply(long long n_items, const float4* packed, const float* x, float
   return cudaGetLastError();
 }
 
+int wt_smem(int S) { return wt_smem_per_warp<N>(S); }
+
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
                       Sh::BFORM ? 1 : 0, steps_per_trip<M, N>() == 3 ? 8 : 6, 1,   // refill threshold K (swept on B200, profiles/r1/solve_variants.txt)
-                      class_index, occupancy, pack, solve, classify, apply};
+                      wt_smem, class_index, occupancy, pack, solve, classify, apply};
 }  // namespace
 
 #define SSHOPM_CAT2(a, b, c) get_launchers_##a##_##b

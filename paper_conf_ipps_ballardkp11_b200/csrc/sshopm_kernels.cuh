@@ -620,6 +620,7 @@ struct SolveParams {
   int S;
   FastDiv divS;
   int s_log2;                // log2(S) if S is a power of two, else -1
+  uint32_t s_mask;           // S - 1 (used when S is a power of two)
   float alpha, tol;
   const float* alpha_t;      // SHIFT == 3: per-tensor shift [N] (from the pack kernel)
   int maxit;
@@ -761,7 +762,7 @@ sshopm_solve_kernel(const SolveParams p) {
         uint32_t s;                                        // its start
         if (p.s_log2 >= 0) {                               // S a power of two (the paper's 128): shift and mask
           tv = item >> p.s_log2;
-          s = (uint32_t)item & (S_ - 1u);
+          s = (uint32_t)item & p.s_mask;
         } else {
           const uint32_t vq = fast_div(t, p.divS);
           s = t - vq * S_;
@@ -929,7 +930,7 @@ sshopm_solve_lean_kernel(const SolveParams p) {
       uint32_t s;
       if (p.s_log2 >= 0) {                               // S a power of two (the paper's 128): shift and mask
         tv = item >> p.s_log2;
-        s = (uint32_t)item & (S_ - 1u);
+        s = (uint32_t)item & p.s_mask;
       } else if constexpr (WIDE) {
         tv = item / S_;
         s = (uint32_t)(item - tv * S_);
@@ -1269,5 +1270,7 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
     out_lam[i] = lam;
   }
 }
+
+#include "sshopm_wt.cuh"
 
 }  // namespace sshopm

@@ -368,6 +368,49 @@ def test_fused_vs_oracle(dev):
     assert np.array_equal(dd[3][same], om2[same])
 
 
+@pytest.mark.parametrize("m,n,V,S,alpha,maxit", [(4, 3, 3000, 128, 0.0, 100), (4, 3, 777, 100, 0.0, 100),
+                                                  (6, 3, 300, 128, 0.25, 100), (4, 6, 100, 64, 0.0, 100),
+                                                  (3, 3, 200, 128, 1.0, 100), (4, 3, 5, 7, 0.0, 100),
+                                                  (4, 3, 2000, 128, 0.0, 3000)])
+def test_schedule7_bitwise(dev, m, n, V, S, alpha, maxit):
+    """Warp-tensor pipeline (schedule 7): raw outputs bitwise equal to schedule 1 (same per-lane arithmetic);
+    fused (clustering from the staging) and records-only forms give the two-pass records bit for bit."""
+    ent = syn.gen_voxels(m, n, 40, V, 4) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 4)
+    if maxit > 1000:
+        ent[::40] = syn.gen_uniform_tensors(m, n, V // 40, 9)      # slow lanes: tensors held open for long
+    st = syn.gen_starts(S, n, 0)
+    a = _solve(dev, m, n, ent, st, alpha, 1e-6, maxit, schedule=1)
+    b = _solve(dev, m, n, ent, st, alpha, 1e-6, maxit, schedule=7)
+    for u, v in zip(a, b):
+        assert np.array_equal(u, v)
+    ra, da = _two_pass(dev, m, n, ent, st, alpha, 1e-6, maxit, 1e-2, 0.05, 4)
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    rb, db = s.solve_dedup(e, t, alpha, 1e-6, maxit, 1e-2, 0.05, 4, schedule=7, fused=True)
+    rc, dc = s.solve_dedup(e, t, alpha, 1e-6, maxit, 1e-2, 0.05, 4, records_only=True)
+    torch.cuda.synchronize()
+    for u, v in zip(ra + da, [x.cpu().numpy() for x in rb + db]):
+        assert np.array_equal(u, v)
+    for u, v in zip(da, [x.cpu().numpy() for x in dc]):
+        assert np.array_equal(u, v)
+
+
+def test_records_only_overflow(dev):
+    """Records-only path with tensors of more than 32 clusters (tight tolerances on unstructured odd-m tensors):
+    those tensors take the raw-output + list-kernel route; records equal the two-pass form."""
+    m, n, V, S = 3, 3, 64, 128
+    ent = syn.gen_uniform_tensors(m, n, V, 2)
+    st = syn.gen_starts(S, n, 1)
+    ra, da = _two_pass(dev, m, n, ent, st, 1.0, 1e-6, 100, 1e-7, 1e-6, 8)
+    assert (da[0] > 32).any()                                    # some tensors overflow the register form
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    rc, dc = s.solve_dedup(e, t, 1.0, 1e-6, 100, 1e-7, 1e-6, 8, records_only=True)
+    torch.cuda.synchronize()
+    for u, v in zip(da, [x.cpu().numpy() for x in dc]):
+        assert np.array_equal(u, v)
+
+
 def test_plain_sshopm_solve_entry_point(dev):
     """sshopm_solve itself: library defaults and its own cudaMallocAsync workspace, data on
     the GPU; bitwise equal to sshopm_solve_ex and within the parity contract."""

@@ -1,7 +1,7 @@
 """Small runs of every solve / dedup path for compute-sanitizer (memcheck, racecheck, synccheck, initcheck):
     compute-sanitizer --tool racecheck python tools/sanitize_run.py <case>
-cases: two_pass (C1 tensors x 128 starts, default schedule: pack + lean solve + dedup), legacy (schedule 6),
-tpl (schedule 2), fused (fuse_dedup = 1: in-kernel ring + list kernel, forced overflow), blocked ((4,10),
+cases: two_pass (C1 tensors x 128 starts, default schedule 1: pack + solve + dedup), lean (schedule 6),
+tpl (schedule 2), wt / wt_records (schedule 7 raw / fused + records-only), fused (fuse_dedup = 1: in-kernel ring + list kernel, forced overflow), blocked ((4,10),
 V = 6, schedule 5, two tensor buffers per warp), general (schedule 3), classify, run_host."""
 import os
 import sys
@@ -21,7 +21,7 @@ def t(a):
     return torch.from_numpy(np.ascontiguousarray(a)).to(dev)
 
 
-if case in ("two_pass", "legacy", "tpl", "fused", "classify"):
+if case in ("two_pass", "legacy", "tpl", "fused", "classify", "lean", "wt", "wt_records"):
     V = 1024 if case != "fused" else 2000
     ent = syn.gen_voxels(4, 3, 0, V, 0)
     if case == "fused":
@@ -30,8 +30,11 @@ if case in ("two_pass", "legacy", "tpl", "fused", "classify"):
     s = sh.Solver(4, 3)
     if case == "fused":
         s.solve_dedup(t(ent), t(st), 0.0, 1e-6, 1000, 1e-2, 0.05, 4, fused=True)
+    elif case == "wt_records":
+        s.solve_dedup(t(ent), t(st), 0.0, 1e-6, 100, 1e-2, 0.05, 4, records_only=True)
+        s.solve_dedup(t(ent), t(st), 0.0, 1e-6, 100, 1e-2, 0.05, 4, schedule=7, fused=True)
     else:
-        sched = {"two_pass": 0, "legacy": 6, "tpl": 2, "classify": 0}[case]
+        sched = {"two_pass": 0, "legacy": 1, "lean": 6, "tpl": 2, "classify": 0, "wt": 7}[case]
         lam, x, it, cv = s.solve(t(ent), t(st), 0.0, 1e-6, 100, schedule=sched)
         cnt, cl, cx, mu, rp = s.dedup(lam, x, cv, 1e-2, 0.05, 8)
         if case == "classify":
