@@ -110,12 +110,16 @@ struct Shape {
 // State layout of x (see xget below): slot of component i.
 #ifndef SSHOPM_43_FORM
 #define SSHOPM_43_FORM 2   // (4,3) step: 2 = (x0,x1),(x2,x1) layout, 8 FMUL2 monomials, scalar FFMA contraction (default:
-                           // C2 4.26 ms); 1 = natural layout, (g0,g1) FFMA2 + g2 FFMA (4.44); 0 = X02 layout, scalar (4.43)
+                           // C2 4.26 ms); 1 = natural layout, (g0,g1) FFMA2 + g2 FFMA (4.44); 0 = X02 layout, scalar (4.43);
+                           // 3 = form 2 without the (x1,x2) moves (4.26); 4 = all scalar (4.79).  DESIGN.md "Round 2".
 #endif
 template <int M, int N>
 struct X02 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 0); };
 template <int M, int N>
 struct N43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 1); };
+// form 4: natural layout, every FP32 operation scalar (FMUL / FFMA / FADD only: no packed FP32 in the step)
+template <int M, int N>
+struct S43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 4); };
 // form 2: the round-1 layout, x held as (x0, x1), (x2, x1) (slot 3 duplicates x1), monomials as 8 FMUL2
 template <int M, int N>
 struct X21 { static constexpr bool v = (M == 4 && N == 3 && (SSHOPM_43_FORM == 2 || SSHOPM_43_FORM == 3)); };
@@ -443,6 +447,24 @@ __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&m
 }
 #endif
 
+// (4,3), form 4: all-scalar evaluation (16 FMUL monomials, 30 FFMA, lambda as an FMA chain).
+__device__ __forceinline__ float eval43s(const Coefs<4, 3>& cf, float x0, float x1, float x2, float& g0, float& g1,
+                                         float& g2) {
+  const float d00 = x0 * x0, d01 = x0 * x1, d02 = x0 * x2, d11 = x1 * x1, d12 = x1 * x2, d22 = x2 * x2;
+  const float mq[10] = {x0 * d00, x0 * d01, x0 * d02, x0 * d11, x0 * d12, x0 * d22, x1 * d11, x1 * d12, x1 * d22,
+                        x2 * d22};
+  g0 = cf.template word<0>() * mq[0];
+  g1 = cf.template word<1>() * mq[0];
+  g2 = cf.template word<20>() * mq[0];
+  static_for<9>([&](auto qq) {
+    constexpr int q = decltype(qq)::value + 1;
+    g0 = fmaf(cf.template word<2 * q>(), mq[q], g0);
+    g1 = fmaf(cf.template word<2 * q + 1>(), mq[q], g1);
+    g2 = fmaf(cf.template word<20 + q>(), mq[q], g2);
+  });
+  return fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
+}
+
 // (4,3), natural layout (x0, x1 | x2): monomials from 7 FMUL2 + 2 FMUL; Eq. 6 as (g0, g1) FFMA2 with the
 // monomial broadcast plus g2 scalar FFMA on the same monomial (q outer).
 __device__ __forceinline__ float eval43n(const Coefs<4, 3>& cf, const float2 (&xs)[2], float2& g01, float& g2) {
@@ -521,6 +543,29 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
     if (!stop) {
       xs[0] = __fmul2_rn(f2(h0, h2), bc(r));
       xs[1].x = h1 * r;
+      lamp = lam;
+      ++k;
+    }
+    return;
+  } else if constexpr (S43<M, N>::v) {
+    const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
+    float g0, g1, g2;
+    lam = eval43s(cf, x0, x1, x2, g0, g1, g2);
+    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
+    float h0, h1, h2;
+    if constexpr (SHIFT == 0) { h0 = g0; h1 = g1; h2 = g2; }
+    else if constexpr (SHIFT == 1) { h0 = fmaf(alpha, x0, g0); h1 = fmaf(alpha, x1, g1); h2 = fmaf(alpha, x2, g2); }
+    else if constexpr (SHIFT == 2) { h0 = fmaf(alpha, x0, -g0); h1 = fmaf(alpha, x1, -g1); h2 = fmaf(alpha, x2, -g2); }
+    else { h0 = fmaf(la, x0, g0 * ls); h1 = fmaf(la, x1, g1 * ls); h2 = fmaf(la, x2, g2 * ls); }
+    const float nn = fmaf(h2, h2, fmaf(h1, h1, h0 * h0));
+    const bool deg = !(nn >= 1.17549435e-38f);
+    if constexpr (KIDLE) stop = conv | (k >= maxit) | deg;
+    else stop = (!has) | conv | (k >= maxit) | deg;
+    const float r = rsqrt_ftz(nn);
+    if (!stop) {
+      xs[0].x = h0 * r;
+      xs[0].y = h1 * r;
+      xs[1].x = h2 * r;
       lamp = lam;
       ++k;
     }
@@ -1243,7 +1288,13 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
     }
     if constexpr (X21<M, N>::v) xs[1].y = xs[0].y;
     float lam;
-    if constexpr (N43<M, N>::v) {
+    if constexpr (S43<M, N>::v) {
+      float g0, g1, g2;
+      lam = eval43s(cf, xs[0].x, xs[0].y, xs[1].x, g0, g1, g2);
+      out_g[i * N + 0] = g0;
+      out_g[i * N + 1] = g1;
+      out_g[i * N + 2] = g2;
+    } else if constexpr (N43<M, N>::v) {
       float2 g01;
       float g2;
       lam = eval43n(cf, xs, g01, g2);
