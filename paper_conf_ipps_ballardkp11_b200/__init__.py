@@ -296,10 +296,11 @@ class Solver:
 
     def solve_dedup(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, lam_tol=1e-2, ang_tol=0.05, kmax=8,
                     out=None, dedup_out=None, refill_threshold=0, ctas_per_sm=0, total_iters=None, stream=None,
-                    schedule=0, fused=False, records_only=False):
+                    schedule=0, fused=False, records_only=False, warp_specialized=False):
         """Fused solve + dedup (sshopm_solve_dedup).  Returns (raw outputs, dedup outputs) as in solve() / dedup().
         fused: cluster inside the solve kernel (schedule 1 ring, or schedule 7 staging).  records_only: the
-        schedule-7 pipeline clusters in-kernel and leaves the raw outputs unwritten (they are scratch)."""
+        schedule-7 pipeline clusters in-kernel and leaves the raw outputs unwritten (they are scratch).
+        warp_specialized: one warp per CTA of the solve kernel clusters the chunks the other seven complete."""
         torch = _torch()
         N, S = int(entries.shape[0]), int(starts.shape[0])
         pe = _dev(entries, torch.float32, (N, self.U), "entries")
@@ -325,7 +326,7 @@ class Solver:
                  _dev(orp, torch.int32, (N, kmax), "out_rep"))
         wsp, wsb = self._workspace(N, S, dev, stream) if N > 0 else (None, 0)
         opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule),
-                     2 if records_only else (1 if fused else 0))
+                     3 if warp_specialized else (2 if records_only else (1 if fused else 0)))
         alpha = self._alpha_opts(alpha, N, opts)
         if total_iters is not None:
             opts.d_total_iters = total_iters.data_ptr()

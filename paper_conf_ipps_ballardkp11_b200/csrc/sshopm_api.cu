@@ -323,14 +323,27 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   // ring + in-kernel clustering push the register-capped solve into spills.
   int fused = 0;                                         // 0 none, 1 shared-memory dedup, 2 register dedup
   int smem = 0;
-  const bool fregs = dd && S == 128 && ((uintptr_t)d_out_lambda % 16 == 0) && ((uintptr_t)d_out_x % 16 == 0) &&
+#ifndef SSHOPM_FUSED_REGS
+#define SSHOPM_FUSED_REGS 1
+#endif
+  const bool fregs = SSHOPM_FUSED_REGS && dd && S == 128 && ((uintptr_t)d_out_lambda % 16 == 0) && ((uintptr_t)d_out_x % 16 == 0) &&
                      ((uintptr_t)d_out_converged % 4 == 0);
   if (dd && (schedule == 1 || schedule == 6) && S <= 1024 && opts && opts->fuse_dedup == 1) {
     const int fs = 8 * fused_smem_words(S, L->n, fregs) * 4;
     int fb = 0;
-    if (fs <= 200 * 1024 && L->occupancy(shift, wide, schedule, fregs ? 2 : 1, fs, &fb) == cudaSuccess && fb >= bps) {
+    if (fs <= 200 * 1024 && L->occupancy(shift, wide, 1, fregs ? 2 : 1, fs, &fb) == cudaSuccess && fb >= bps) {
       fused = fregs ? 2 : 1;
       smem = fs;
+    }
+  }
+  // warp-specialised fused dedup (opts->fuse_dedup = 3): 7 solve warps + 1 dedup warp per CTA
+  if (dd && (schedule == 1 || schedule == 6) && S <= 1024 && opts && opts->fuse_dedup == 3) {
+    const int fs = ws_smem_words(S, L->n) * 4;
+    int fb = 0;
+    if (fs <= 200 * 1024 && L->occupancy(shift, wide, 1, 3, fs, &fb) == cudaSuccess && fb >= 1) {
+      fused = 3;
+      smem = fs;
+      bps = fb;
     }
   }
   if (fused) schedule = 1;                                       // the fused ring lives in the schedule-1 kernel

@@ -24,12 +24,15 @@ const void* wt_fn() { return reinterpret_cast<const void*>(sshopm_solve_wt_kerne
 template <int SH, bool W, int F>
 cudaError_t occ2(int schedule, int smem, int* bps) {
   if (schedule == 7) {   // warp-tensor pipeline: F = MODE (0 raw, 1 records only, 2 both); smem = staging bytes
-    const void* fn = wt_fn<SH, F>();
-    if (smem > 48 * 1024) {
-      cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-      if (e != cudaSuccess) return e;
+    if constexpr (F <= 2) {
+      const void* fn = wt_fn<SH, F>();
+      if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+      }
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, fn, 256, smem);
     }
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, fn, 256, smem);
+    return cudaErrorInvalidValue;
   }
   if constexpr (SH == 3) {
     if (schedule == 2) return cudaErrorInvalidValue;         // per-tensor alpha: schedule 1 only
@@ -42,6 +45,7 @@ cudaError_t occ2(int schedule, int smem, int* bps) {
 }
 template <int SH, bool W>
 cudaError_t occ1(int schedule, int fused, int smem, int* bps) {
+  if (fused == 3) return occ2<SH, W, 3>(schedule, smem, bps);
   return fused == 2 ? occ2<SH, W, 2>(schedule, smem, bps) : fused == 1 ? occ2<SH, W, 1>(schedule, smem, bps)
                     : occ2<SH, W, 0>(schedule, smem, bps);
 }
@@ -61,7 +65,7 @@ cudaError_t occupancy(int shift, bool wide, int schedule, int fused, int smem, i
 template <int SH, bool W, int F>
 cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaStream_t st) {
   if (schedule == 7) {
-    if constexpr (!W) {
+    if constexpr (!W && F <= 2) {
       if (smem > 48 * 1024) {
         cudaError_t e = cudaFuncSetAttribute(sshopm_solve_wt_kernel<M, N, SH, F>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -82,12 +86,16 @@ cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaS
       cudaError_t e = cudaFuncSetAttribute(sshopm_solve_kernel<M, N, SH, W, F>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       if (e != cudaSuccess) return e;
     }
-    sshopm_solve_kernel<M, N, SH, W, F><<<grid, 256, smem, st>>>(p);
+#ifndef SSHOPM_SOLVE_THREADS
+#define SSHOPM_SOLVE_THREADS 256
+#endif
+    sshopm_solve_kernel<M, N, SH, W, F><<<grid, SSHOPM_SOLVE_THREADS, smem, st>>>(p);
   }
   return cudaGetLastError();
 }
 template <int SH, bool W>
 cudaError_t solve1(const SolveParams& p, int schedule, int fused, int grid, int smem, cudaStream_t st) {
+  if (fused == 3) return solve2<SH, W, 3>(p, schedule, grid, smem, st);
   return fused == 2 ? solve2<SH, W, 2>(p, schedule, grid, smem, st) : fused == 1 ? solve2<SH, W, 1>(p, schedule, grid, smem, st)
                     : solve2<SH, W, 0>(p, schedule, grid, smem, st);
 }

@@ -681,6 +681,15 @@ constexpr int kFusedRing = 16;   // open-chunk ring per warp (fused solve -> ded
 __host__ __device__ constexpr int fused_smem_words(int S, int n, bool regs) {
   return 3 * kFusedRing + (regs ? 0 : dedup_smem_words(S, n));
 }
+// Fused mode 3 (warp-specialised): warps 0..6 solve, warp 7 clusters the chunks they complete.  Shared
+// memory: 8 open-chunk rings, a CTA queue of completed chunks (kWsQueue slots + head, tail, finished),
+// the dedup warp's fallback staging (tensors with > 32 clusters, or S != 128).
+constexpr int kWsQueue = 64;     // power of two
+constexpr int kWsSolveWarps = 7;
+constexpr unsigned int kWsEmpty = 0xffffffffu;
+__host__ __device__ constexpr int ws_smem_words(int S, int n) {
+  return 8 * 3 * kFusedRing + kWsQueue + 4 + dedup_smem_words(S, n);
+}
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t r;
@@ -698,6 +707,7 @@ template <int M, int N, int SHIFT, bool WIDE, int FUSED_MODE>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
   constexpr bool FUSED = FUSED_MODE != 0;        // 1: shared-memory dedup (any S <= 1024), 2: register dedup (S = 128)
+  constexpr bool WS = FUSED_MODE == 3;           // 3: warp-specialised (a dedup warp per CTA consumes completed chunks)
   constexpr int STEPS = steps_per_trip<M, N>();        // SS-HOPM steps between refill checks
   using S = Shape<M, N>;
   using Idx = typename std::conditional<WIDE, long long, uint32_t>::type;
@@ -713,7 +723,46 @@ sshopm_solve_kernel(const SolveParams p) {
 
   // fused dedup: per-warp open-chunk ring + dedup staging in shared memory
   extern __shared__ int fsm[];
-  int* r_seq = fsm + (threadIdx.x >> 5) * fused_smem_words(p.S, N, FUSED_MODE == 2);
+  int* r_seq = fsm + (threadIdx.x >> 5) * (WS ? 3 * kFusedRing : fused_smem_words(p.S, N, FUSED_MODE == 2));
+  unsigned int* wq = reinterpret_cast<unsigned int*>(fsm + 8 * 3 * kFusedRing);   // WS: [kWsQueue] + head, tail, finished
+  if constexpr (WS) {
+    for (int i = threadIdx.x; i < kWsQueue; i += blockDim.x) wq[i] = kWsEmpty;
+    if (threadIdx.x == 0) { wq[kWsQueue] = 0u; wq[kWsQueue + 1] = 0u; wq[kWsQueue + 2] = 0u; }
+    __syncthreads();
+    if ((threadIdx.x >> 5) == kWsSolveWarps) {     // ---- the dedup warp ----
+      volatile unsigned int* vq = wq;
+      float* st = reinterpret_cast<float*>(wq + kWsQueue + 4);
+      float* s_lam = st;
+      float* s_x = s_lam + p.S;
+      int* s_cid = reinterpret_cast<int*>(s_x + (size_t)p.S * N);
+      float* c_lam = reinterpret_cast<float*>(s_cid + p.S);
+      int* c_rep = reinterpret_cast<int*>(c_lam + p.S);
+      int* c_mult = c_rep + p.S;
+      unsigned int h = 0;
+      for (;;) {
+        if (h == vq[kWsQueue + 1]) {
+          if (vq[kWsQueue + 2] == (unsigned int)kWsSolveWarps && h == vq[kWsQueue + 1]) break;
+          __nanosleep(200);
+          continue;
+        }
+        unsigned int ch;
+        while ((ch = vq[h & (kWsQueue - 1)]) == kWsEmpty) {}   // slot reserved, chunk index not yet written
+        __syncwarp();
+        if (lane == 0) { vq[h & (kWsQueue - 1)] = kWsEmpty; vq[kWsQueue] = h + 1; }
+        ++h;
+        __threadfence_block();                      // acquire: the producer fenced its raw-output stores
+        const long long v0 = (long long)ch * p.chunk_tensors;
+        const long long v1 = min(p.n_tensors, v0 + p.chunk_tensors);
+#pragma unroll 1
+        for (long long v = v0; v < v1; ++v) {
+          bool ok = false;
+          if (p.fused_regs) ok = warp_dedup128_regs<N, (M % 2) == 0>(p.dd, v, lane);
+          if (!ok) warp_dedup_tensor<N, (M % 2) == 0>(p.dd, v, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
+        }
+      }
+      return;
+    }
+  }
   unsigned int* r_chunk = reinterpret_cast<unsigned int*>(r_seq + kFusedRing);
   int* r_rem = r_seq + 2 * kFusedRing;
   float* d_lam = reinterpret_cast<float*>(r_seq + 3 * kFusedRing);
@@ -843,7 +892,35 @@ sshopm_solve_kernel(const SolveParams p) {
           c_next += cnt;
         }
       }
-      if constexpr (FUSED) {
+      if constexpr (WS) {
+        uint32_t dmask = __ballot_sync(FULL, chunk_done);
+        if (dmask) {                                       // publish the completed chunks to the dedup warp
+          __threadfence_block();                           // release: this warp's raw-output stores first
+          __syncwarp();
+          do {
+            const int src = __ffs(dmask) - 1;
+            dmask &= dmask - 1;
+            const int slot = __shfl_sync(FULL, done_slot, src);
+            if (lane == 0) {
+              volatile unsigned int* vq = wq;
+              const unsigned int ch = r_chunk[slot];
+              unsigned int t = vq[kWsQueue + 1];
+              bool queued = false;
+              for (;;) {                                   // reserve a queue slot unless the queue is full
+                if (t - vq[kWsQueue] >= (unsigned int)kWsQueue) break;
+                const unsigned int o = atomicCAS(wq + kWsQueue + 1, t, t + 1);
+                if (o == t) { queued = true; break; }
+                t = o;
+              }
+              if (queued) vq[t & (kWsQueue - 1)] = ch;
+              else p.ovf_list[atomicAdd(p.ovf_count, 1u)] = ch;   // full: clustered by the list kernel
+              r_seq[slot] = -1;
+            }
+            __syncwarp();
+          } while (dmask);
+        }
+      }
+      if constexpr (FUSED && !WS) {
         uint32_t dmask = __ballot_sync(FULL, chunk_done);
         if (dmask) {                                       // cluster the completed chunks' tensors now (L2-hot)
           __threadfence_block();
@@ -882,6 +959,10 @@ sshopm_solve_kernel(const SolveParams p) {
     for (int rep = 0; rep < STEPS; ++rep)
       sshopm_step<M, N, SHIFT, true>(cf, xs, lam, lamp, k, conv, stop, has, alpha, la, ls, tol, maxit);
     __syncwarp();
+  }
+  if constexpr (WS) {                                      // every chunk of this warp has been published
+    __threadfence_block();
+    if (lane == 0) atomicAdd(wq + kWsQueue + 2, 1u);
   }
 
   if (p.total_iters) {

@@ -426,6 +426,25 @@ def test_plain_sshopm_solve_entry_point(dev):
     _assert_parity(PR.solve_parity(ent, st, m, n, 0.0, 1e-6, 100, tuple(a)))
 
 
+@pytest.mark.parametrize("m,n,V,S,alpha,maxit", [(4, 3, 3000, 128, 0.0, 100), (4, 3, 777, 100, 0.0, 100),
+                                                  (6, 3, 500, 128, 0.25, 100), (3, 3, 400, 64, 1.0, 100),
+                                                  (4, 3, 2000, 128, 0.0, 3000)])
+def test_fused_warp_specialised_equals_two_pass(dev, m, n, V, S, alpha, maxit):
+    """Fused mode 3 (one dedup warp per CTA consumes the chunks the solve warps complete): raw and dedup
+    outputs bit for bit those of the two-pass form, including slow tensors that overflow the rings."""
+    ent = syn.gen_voxels(m, n, 900, V, 1) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 1)
+    if maxit > 1000:
+        ent[::40] = syn.gen_uniform_tensors(m, n, V // 40, 9)
+    st = syn.gen_starts(S, n, 3)
+    ra, da = _two_pass(dev, m, n, ent, st, alpha, 1e-6, maxit, 1e-2, 0.05, 4)
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    rb, db = s.solve_dedup(e, t, alpha, 1e-6, maxit, 1e-2, 0.05, 4, warp_specialized=True)
+    torch.cuda.synchronize()
+    for a, b in zip(ra + da, [x.cpu().numpy() for x in rb + db]):
+        assert np.array_equal(a, b)
+
+
 def test_fused_ring_overflow(dev):
     """Chunks held open for thousands of steps by slow lanes overflow the per-warp ring; the
     follow-up list kernel must still cluster them (results identical to the two-pass form)."""
