@@ -538,6 +538,7 @@ def main():
         "ms_solve_per_step": solve_ms / a.steps,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tflops, "unit": "TFLOP/s",
                      "frac": achieved / peak_tflops, "traffic": traffic,
+                     "frac_updates_only": Fx * iters_local * a.steps / (solve_ms / 1e3) / 1e12 / peak_tflops,
                      "kernel": f"sshopm_solve_kernel<{m},{n}>",
                      "peak_basis": f"{sms} SM x 128 FP32 lanes x 2 x {fmax:.0f} MHz (sm_max_mhz)",
                      "flops_per_update": Fx, "flops_lambda0_eval": Fe,
@@ -546,7 +547,8 @@ def main():
                      "executed_frac_ncu": (exec_gflop * 1e9 / (solve_ms / a.steps / 1e3) / 1e12 / peak_tflops
                                            if exec_gflop and world == 1 else None),
                      "flops_note": "algorithmic FP32 flops per launch = flops_per_update x sum(iters) + flops_lambda0_eval x N*S "
-                                   "(update: monomials + 2*T1 + lambda + shift + norm + scale; lambda_0: monomials + 2*T1 + lambda; DESIGN.md 7)"},
+                                   "(update: monomials + 2*T1 + lambda + shift + norm + scale; lambda_0: monomials + 2*T1 + lambda; DESIGN.md 7); "
+                                   "frac_updates_only counts the updates alone (lambda_0 evaluations as free work)"},
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,

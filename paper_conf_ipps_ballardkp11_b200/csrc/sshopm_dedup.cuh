@@ -236,9 +236,9 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
   float n2[SPL];
 #pragma unroll
   for (int c = 0; c < SPL; ++c) n2[c] = dd_norm2<N>(xs[c]);
-  uint32_t un = 0;                                   // unassigned converged starts (bit c = start 4*lane + c)
-#pragma unroll
-  for (int c = 0; c < SPL; ++c) un |= ((r.conv >> (8 * c)) & 0xffu) ? (1u << c) : 0u;
+  // unassigned converged starts (bit c = start 4*lane + c): byte c nonzero -> bit c
+  const uint32_t nz = __vcmpne4(r.conv, 0u) & 0x08040201u;
+  uint32_t un = (nz | (nz >> 8) | (nz >> 16) | (nz >> 24)) & 0xfu;
   if constexpr (STAGE) {
     reinterpret_cast<float4*>(stage)[lane] = r.lam;
 #pragma unroll
@@ -298,20 +298,25 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
   }
   if (lane == 0) p.out_count[v] = ncl;
   const long long ob = v * p.kmax;
-  if (lane < ncl && rank < p.kmax) {
-    p.out_lambda[ob + rank] = my_lam;
+  // one store pass: lane c < ncl writes cluster c at its rank (if ranked within kmax); lanes ncl..kmax-1
+  // write the empty slots ncl..kmax-1 (ranks of the ncl clusters are exactly 0..ncl-1)
+  const bool mine = lane < ncl;
+  const int slot = mine ? rank : lane;
+  if (mine ? (rank < p.kmax) : (lane < p.kmax)) {
+    p.out_lambda[ob + slot] = mine ? my_lam : 0.f;
 #pragma unroll
-    for (int j = 0; j < N; ++j) p.out_x[(ob + rank) * N + j] = my_x[j];
-    p.out_mult[ob + rank] = my_mult;
-    if (p.out_rep) p.out_rep[ob + rank] = my_rep;
+    for (int j = 0; j < N; ++j) p.out_x[(ob + slot) * N + j] = mine ? my_x[j] : 0.f;
+    p.out_mult[ob + slot] = mine ? my_mult : 0;
+    if (p.out_rep) p.out_rep[ob + slot] = mine ? my_rep : -1;
   }
 #pragma unroll 1
-  for (int slot = ncl + lane; slot < p.kmax; slot += 32) {
-    p.out_lambda[ob + slot] = 0.f;
+  for (int sl = 32 + lane; sl < p.kmax; sl += 32) {  // kmax > 32 only
+    if (sl < ncl) continue;
+    p.out_lambda[ob + sl] = 0.f;
 #pragma unroll
-    for (int j = 0; j < N; ++j) p.out_x[(ob + slot) * N + j] = 0.f;
-    p.out_mult[ob + slot] = 0;
-    if (p.out_rep) p.out_rep[ob + slot] = -1;
+    for (int j = 0; j < N; ++j) p.out_x[(ob + sl) * N + j] = 0.f;
+    p.out_mult[ob + sl] = 0;
+    if (p.out_rep) p.out_rep[ob + sl] = -1;
   }
   if constexpr (STAGE) __syncwarp();                 // the stage is rewritten by the next tensor
   return true;
@@ -329,20 +334,27 @@ __global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams 
   float* gen = smem + (size_t)(blockDim.x >> 5) * 128 * (N + 1) + (size_t)wib * dedup_smem_words(128, N);
   const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
   long long v = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
-  DedupRegs<N> nx;
-  if (v < p.n_tensors) dedup_load<N>(nx, p, v, lane, true);
-  for (; v < p.n_tensors; v += warps) {
-    const DedupRegs<N> cur = nx;
-    if (v + warps < p.n_tensors) dedup_load<N>(nx, p, v + warps, lane, true);   // prefetch
-    if (!dedup128_regs<N, EVEN, true>(p, v, lane, cur, stage)) {
+  auto run = [&](const DedupRegs<N>& cur, long long t) {
+    if (!dedup128_regs<N, EVEN, true>(p, t, lane, cur, stage)) {
       float* s_lam = gen;
       float* s_x = s_lam + 128;
       int* s_cid = reinterpret_cast<int*>(s_x + 128 * N);
       float* c_lam = reinterpret_cast<float*>(s_cid + 128);
       int* c_rep = reinterpret_cast<int*>(c_lam + 128);
       int* c_mult = c_rep + 128;
-      warp_dedup_tensor<N, EVEN>(p, v, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
+      warp_dedup_tensor<N, EVEN>(p, t, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
     }
+  };
+  // two register buffers used alternately (the next tensor is loaded while the current one is clustered,
+  // without copying the buffer: 17 register moves per tensor fewer than a single prefetch buffer)
+  DedupRegs<N> a, b;
+  if (v < p.n_tensors) dedup_load<N>(a, p, v, lane, true);
+  for (; v < p.n_tensors; v += 2 * warps) {
+    if (v + warps < p.n_tensors) dedup_load<N>(b, p, v + warps, lane, true);
+    run(a, v);
+    if (v + warps >= p.n_tensors) break;
+    if (v + 2 * warps < p.n_tensors) dedup_load<N>(a, p, v + 2 * warps, lane, true);
+    run(b, v + warps);
   }
 }
 // shared-memory bytes per warp of sshopm_dedup128_kernel (stage + fallback staging)

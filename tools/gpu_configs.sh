@@ -1,4 +1,5 @@
 #!/bin/bash
+TAG=${TAG:-r2}
 # Bench lines for every config (C2 default first) + C2 launch list and solve-kernel ncu capture.
 OUT=gpurun_out/${1:-cfg}; mkdir -p $OUT
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $OUT/smi.txt 2>&1
