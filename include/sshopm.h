@@ -114,8 +114,9 @@ typedef struct {
   size_t workspace_bytes;          /* its size; a too-small or misaligned workspace returns EINVAL */
   int schedule;                    /* 0 default, 1 = item per lane (warps claim chunks of whole tensors),
                                       2 = tensor per lane (a lane walks one tensor's starts), 6 = item per lane
-                                      with a branch-free predicated refill and one chunk in flight (measured
-                                      slower on B200, kept for comparison); results identical.
+                                      with a branch-free predicated refill and one chunk in flight, 7 = warp-
+                                      tensor pipeline (shared-memory staging, coalesced flushes); 6 and 7 are
+                                      measured slower on B200 and kept for comparison; results identical.
                                       Table-driven general kernel (the only path for (m, n) without a compiled
                                       kernel): 5 = blocked (default): warp per tensor, the
                                       tensor's coefficient-folded rows once per warp in shared memory, blocks of
@@ -124,8 +125,9 @@ typedef struct {
                                       thread per start (the paper's mapping); 3-5 also force the
                                       table-driven path on compiled shapes (5 returns EUNSUPPORTED if its
                                       shared memory does not fit; the default then falls back to 3, then 4). */
-  int fuse_dedup;                  /* sshopm_solve_dedup only: 1 = cluster inside the solve kernel (fused),
-                                      0 = default (two passes; faster on B200); results identical */
+  int fuse_dedup;                  /* sshopm_solve_dedup only: 0 = default (two passes; fastest on B200),
+                                      1 = solve warps cluster their chunks, 3 = one dedup warp per CTA,
+                                      2 = records only (schedule 7 pipeline); results identical */
   int alpha_mode;                  /* shift: 0 = the scalar alpha argument (default);
                                       1 = per tensor, d_alpha[N] (device); 2 = per tensor automatic convex shift
                                       alpha_t = +(m-1) sum_{all indices} |a| (>= beta(A): lambda_k nondecreasing,
@@ -155,7 +157,7 @@ int sshopm_solve_ex(sshopm_t h, int64_t N, const float* d_entries, int S, const 
  * (members), d_out_rep[N][kmax] (representative start, -1 in empty slots;
  * d_out_rep may be NULL).  Empty slots: lambda 0, x 0, mult 0.
  * Inputs are sshopm_solve's outputs.  Errors: EINVAL (kmax < 1, negative
- * tolerances, null pointers), EUNSUPPORTED (S > 1024), ECUDA. */
+ * tolerances, null pointers), EUNSUPPORTED (S > 1024 or n > 16), ECUDA. */
 int sshopm_dedup(sshopm_t h, int64_t N, int S,
                  const float* d_lambda, const float* d_x, const uint8_t* d_converged,
                  float lam_tol, float ang_tol, int kmax,
@@ -168,11 +170,16 @@ int sshopm_dedup(sshopm_t h, int64_t N, int S,
  * warp of the solve kernel clusters a chunk of tensors as soon as it has
  * written the chunk's last start (reading the raw outputs back from L2); the
  * few chunks it cannot track are clustered by a small follow-up kernel.
- * Raw outputs are required (they are also the dedup's input).  The fused form
- * is opt-in (opts->fuse_dedup = 1); by default, and whenever the fused form
- * does not apply (schedule 2, or its shared memory would lower occupancy),
- * the two passes run back to back on the stream.  Errors: as sshopm_solve_ex
- * and sshopm_dedup. */
+ * Raw outputs are required (they are also the dedup's input).  The fused forms
+ * are opt-in: opts->fuse_dedup = 1, the solve warps cluster their own chunks;
+ * 3, one warp per CTA clusters the chunks the other seven complete (a CTA
+ * queue in shared memory); 2, records only: the warp-tensor pipeline
+ * (schedule 7) clusters each tensor from its shared-memory staging and writes
+ * raw outputs only for tensors with more than 32 clusters (S = 128; the raw
+ * output arrays are then scratch).  All are measured slower than the two
+ * passes on B200.  By default, and whenever a fused
+ * form does not apply, the two passes run back to back on the stream.
+ * Errors: as sshopm_solve_ex and sshopm_dedup. */
 int sshopm_solve_dedup(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts,
                        float alpha, float tol, int maxit,
                        float* d_out_lambda, float* d_out_x, int32_t* d_out_iters, uint8_t* d_out_converged,

@@ -531,7 +531,7 @@ int make_dedup_params(int n, int64_t N, int S, float lam_tol, float ang_tol, int
   if (S < 1 || kmax < 1 || !(lam_tol >= 0.f) || !(ang_tol >= 0.f) || N < 0) return SSHOPM_EINVAL;
   if (N > 0 && (!d_count || !d_olam || !d_ox || !d_mult)) return SSHOPM_EINVAL;
   if (S > 1024) return SSHOPM_EUNSUPPORTED;
-  if (n > 8) return SSHOPM_EUNSUPPORTED;
+  if (n > 16) return SSHOPM_EUNSUPPORTED;                    // the blocked kernel's largest n
   p->lambda = nullptr;
   p->x = nullptr;
   p->conv = nullptr;
@@ -568,7 +568,7 @@ int launch_dedup(int m, int n, const DedupParams& p, cudaStream_t st) {
   if (p.n_tensors == 0) return SSHOPM_OK;
   if (!p.lambda || !p.x || !p.conv) return SSHOPM_EINVAL;
   const int S = p.S;
-  const bool fast = (S == 128) && ((uintptr_t)p.lambda % 16 == 0) && ((uintptr_t)p.x % 16 == 0) &&
+  const bool fast = (S == 128) && n <= 8 && ((uintptr_t)p.lambda % 16 == 0) && ((uintptr_t)p.x % 16 == 0) &&
                     ((uintptr_t)p.conv % 4 == 0);
   int grid, block, smem;
   int rc = dedup_launch_shape(n, p.n_tensors, S, fast, &grid, &block, &smem);
@@ -580,6 +580,10 @@ int launch_dedup(int m, int n, const DedupParams& p, cudaStream_t st) {
                              : (even ? launch_dedup_t<NN, true>(p, grid, block, smem, st) : launch_dedup_t<NN, false>(p, grid, block, smem, st)); break;
     DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
 #undef DD
+#define DG(NN) case NN: e = even ? launch_dedup_t<NN, true>(p, grid, block, smem, st) \
+                             : launch_dedup_t<NN, false>(p, grid, block, smem, st); break;
+    DG(9) DG(10) DG(11) DG(12) DG(13) DG(14) DG(15) DG(16)
+#undef DG
     default: return SSHOPM_EUNSUPPORTED;
   }
   if (e != cudaSuccess) return cuda_fail(e, "sshopm_dedup: launch");
@@ -609,7 +613,7 @@ int launch_dedup_list(int m, int n, const DedupParams& p, const unsigned int* co
   switch (n) {
 #define DD(NN) case NN: e = even ? launch_list_t<NN, true>(p, count, list, chunk_tensors, grid, block, smem, st) \
                              : launch_list_t<NN, false>(p, count, list, chunk_tensors, grid, block, smem, st); break;
-    DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8)
+    DD(1) DD(2) DD(3) DD(4) DD(5) DD(6) DD(7) DD(8) DD(9) DD(10) DD(11) DD(12) DD(13) DD(14) DD(15) DD(16)
 #undef DD
     default: return SSHOPM_EUNSUPPORTED;
   }

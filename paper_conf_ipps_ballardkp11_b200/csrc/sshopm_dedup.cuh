@@ -236,9 +236,18 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
   float n2[SPL];
 #pragma unroll
   for (int c = 0; c < SPL; ++c) n2[c] = dd_norm2<N>(xs[c]);
+#ifndef SSHOPM_DD_MASK
+#define SSHOPM_DD_MASK 1   // byte-mask unpack of the converged flags (C2: 0.422 -> 0.420 ms)
+#endif
+#if SSHOPM_DD_MASK
   // unassigned converged starts (bit c = start 4*lane + c): byte c nonzero -> bit c
   const uint32_t nz = __vcmpne4(r.conv, 0u) & 0x08040201u;
   uint32_t un = (nz | (nz >> 8) | (nz >> 16) | (nz >> 24)) & 0xfu;
+#else
+  uint32_t un = 0;                                   // unassigned converged starts (bit c = start 4*lane + c)
+#pragma unroll
+  for (int c = 0; c < SPL; ++c) un |= ((r.conv >> (8 * c)) & 0xffu) ? (1u << c) : 0u;
+#endif
   if constexpr (STAGE) {
     reinterpret_cast<float4*>(stage)[lane] = r.lam;
 #pragma unroll
@@ -298,6 +307,10 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
   }
   if (lane == 0) p.out_count[v] = ncl;
   const long long ob = v * p.kmax;
+#ifndef SSHOPM_DD_ONEPASS
+#define SSHOPM_DD_ONEPASS 1   // records and empty slots in one predicated store pass (0.422 -> 0.404 ms)
+#endif
+#if SSHOPM_DD_ONEPASS
   // one store pass: lane c < ncl writes cluster c at its rank (if ranked within kmax); lanes ncl..kmax-1
   // write the empty slots ncl..kmax-1 (ranks of the ncl clusters are exactly 0..ncl-1)
   const bool mine = lane < ncl;
@@ -318,6 +331,23 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
     p.out_mult[ob + sl] = 0;
     if (p.out_rep) p.out_rep[ob + sl] = -1;
   }
+#else
+  if (lane < ncl && rank < p.kmax) {
+    p.out_lambda[ob + rank] = my_lam;
+#pragma unroll
+    for (int j = 0; j < N; ++j) p.out_x[(ob + rank) * N + j] = my_x[j];
+    p.out_mult[ob + rank] = my_mult;
+    if (p.out_rep) p.out_rep[ob + rank] = my_rep;
+  }
+#pragma unroll 1
+  for (int slot = ncl + lane; slot < p.kmax; slot += 32) {
+    p.out_lambda[ob + slot] = 0.f;
+#pragma unroll
+    for (int j = 0; j < N; ++j) p.out_x[(ob + slot) * N + j] = 0.f;
+    p.out_mult[ob + slot] = 0;
+    if (p.out_rep) p.out_rep[ob + slot] = -1;
+  }
+#endif
   if constexpr (STAGE) __syncwarp();                 // the stage is rewritten by the next tensor
   return true;
 }
@@ -345,8 +375,11 @@ __global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams 
       warp_dedup_tensor<N, EVEN>(p, t, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
     }
   };
-  // two register buffers used alternately (the next tensor is loaded while the current one is clustered,
-  // without copying the buffer: 17 register moves per tensor fewer than a single prefetch buffer)
+#ifndef SSHOPM_DD_TWOBUF
+#define SSHOPM_DD_TWOBUF 0   // two alternating prefetch buffers: measured slower (0.463 ms)
+#endif
+#if SSHOPM_DD_TWOBUF
+  // two register buffers used alternately (no copy of the prefetched buffer)
   DedupRegs<N> a, b;
   if (v < p.n_tensors) dedup_load<N>(a, p, v, lane, true);
   for (; v < p.n_tensors; v += 2 * warps) {
@@ -356,6 +389,15 @@ __global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams 
     if (v + 2 * warps < p.n_tensors) dedup_load<N>(a, p, v + 2 * warps, lane, true);
     run(b, v + warps);
   }
+#else
+  DedupRegs<N> nx;
+  if (v < p.n_tensors) dedup_load<N>(nx, p, v, lane, true);
+  for (; v < p.n_tensors; v += warps) {
+    const DedupRegs<N> cur = nx;
+    if (v + warps < p.n_tensors) dedup_load<N>(nx, p, v + warps, lane, true);   // prefetch
+    run(cur, v);
+  }
+#endif
 }
 // shared-memory bytes per warp of sshopm_dedup128_kernel (stage + fallback staging)
 __host__ __device__ constexpr int dedup128_smem_per_warp(int n) { return (128 * (n + 1) + dedup_smem_words(128, n)) * 4; }

@@ -262,6 +262,21 @@ def test_dedup_start_counts(dev, S):
     assert np.array_equal(cl.astype(np.float64), ol) and np.array_equal(cx.astype(np.float64), ox)
 
 
+@pytest.mark.parametrize("m,n,V,S", [(4, 10, 6, 32), (3, 9, 8, 40), (6, 12, 3, 16)])
+def test_dedup_large_n(dev, m, n, V, S):
+    """Dedup for n > 8 (the blocked kernel's shapes): the shared-memory kernel vs the oracle rule on the same
+    per-start results."""
+    ent = syn.gen_voxels(m, n, 0, V, 5) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 5)
+    st = syn.gen_starts(S, n, 4)
+    s = sh.Solver(m, n)
+    alpha = 0.0 if m % 2 == 0 else 2.0
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), alpha, 1e-6, 300)
+    cnt, cl, cx, mu, rp = (t.cpu().numpy() for t in s.dedup(lam, x, cv, 1e-2, 0.05, 6))
+    oc, ol, ox, om, orp = D.dedup(lam.cpu().numpy(), x.cpu().numpy(), cv.cpu().numpy().astype(bool), m, 1e-2, 0.05, 6)
+    assert np.array_equal(cnt, oc) and np.array_equal(rp, orp) and np.array_equal(mu, om)
+    assert np.array_equal(cl.astype(np.float64), ol) and np.array_equal(cx.astype(np.float64), ox)
+
+
 def test_dedup_odd_m(dev):
     m, n = 3, 3
     ent = syn.gen_uniform_tensors(m, n, 128, 1)
