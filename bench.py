@@ -535,6 +535,10 @@ def main():
         "converged_frac": conv_frac,
         "dedup_clusters_hist": {str(k) if k <= KMAX else f">{KMAX}": v for k, v in enumerate(hist)},
         "voxel_solves_frac_of_peak_equiv": vps / (peak_tflops * 1e12 / (F * mean_it * S)),
+        "value_note": "value and voxel_solves_frac_of_peak_equiv use the paper-style flop count (reading R12: "
+                      f"{F} flops per update for ({m},{n}), about 2.8x the FP32 work the kernel executes for (4,3)); "
+                      "they are comparable to the paper's 318 GFLOP/s, not a fraction of peak. The fraction of the FP32 "
+                      "peak is roofline.frac (algorithmic flops) and roofline.executed_frac_ncu (executed flops).",
         "ms_solve_per_step": solve_ms / a.steps,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tflops, "unit": "TFLOP/s",
                      "frac": achieved / peak_tflops, "traffic": traffic,

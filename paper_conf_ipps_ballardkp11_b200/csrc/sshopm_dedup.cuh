@@ -281,11 +281,12 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
     const float rn = dd_norm2<N>(rx);
     const float ltol = p.lam_tol * fmaxf(1.0f, fabsf(rl));
     const float lim2 = ct2 * rn;
-    const int fsel = first - SPL * lane;             // local index of the representative if this lane owns it
+    // The representative matches itself: its (lambda, x) and squared norm are bit-identical copies, so
+    // |dlambda| = 0 and dot = n2 = rn exactly, and cos_tol^2 <= 1 keeps lim2 * n2 <= dot^2 under rounding.
     uint32_t hit = 0;
 #pragma unroll
     for (int c = 0; c < SPL; ++c) {                  // evaluated for every start, masked afterwards (no branches)
-      const bool same = (fsel == c) | dd_same<N, EVEN>(lam[c], xs[c], n2[c], rl, rx, rn, lim2, ltol, p.cos_tol);
+      const bool same = dd_same<N, EVEN>(lam[c], xs[c], n2[c], rl, rx, rn, lim2, ltol, p.cos_tol);
       hit |= same ? (1u << c) : 0u;
     }
     hit &= un;
