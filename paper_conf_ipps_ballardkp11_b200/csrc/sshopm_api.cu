@@ -6,6 +6,7 @@
 // except inside sshopm_run_host (host_pipeline.cu).
 #include <atomic>
 #include <cmath>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -553,7 +554,9 @@ static int dedup_launch_shape(int n, int64_t N, int S, bool fast, int* grid, int
   if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_dedup: no device");
   const int per_warp = fast ? dedup128_smem_per_warp(n) : dedup_smem_words(S, n) * 4;
   int wpb = (96 * 1024) / per_warp;
-  if (wpb > 8) wpb = 8;
+  static const int wmax = [] { const char* v = getenv("SSHOPM_DEDUP_WARPS"); int w = v ? atoi(v) : 8;
+                               return w < 1 ? 1 : (w > 8 ? 8 : w); }();   // warps per dedup CTA (default 8)
+  if (wpb > wmax) wpb = wmax;
   if (wpb < 1) wpb = 1;
   *smem = wpb * per_warp;
   *block = 32 * wpb;
