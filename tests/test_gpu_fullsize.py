@@ -18,7 +18,7 @@ import synthetic as syn  # noqa: E402
 from tests import parity as PR  # noqa: E402
 
 # config -> number of sampled tensors checked against the oracle
-SAMPLES = {"C2": 512, "C2a": 384, "C3": 192, "C4a": 32, "C4b": 128}
+SAMPLES = {"C2": 512, "C2a": 384, "C3": 192, "C4a": 32, "C4b": 128, "C5": 512}
 
 
 @pytest.fixture(scope="module")
@@ -28,8 +28,9 @@ def dev():
     return torch.device("cuda:0")
 
 
-@pytest.mark.parametrize("cfg_name", ["C2", "C2a", "C3", "C4a", "C4b"])
+@pytest.mark.parametrize("cfg_name", ["C2", "C2a", "C3", "C4a", "C4b", "C5"])
 def test_fullsize_sampled_parity(dev, cfg_name):
+    """C5 is the whole 2^23-tensor volume on one GPU (the multi-GPU config's data)."""
     c = syn.CONFIGS[cfg_name]
     m, n, N, S = c["m"], c["n"], c["N"], c["S"]
     ent = syn.gen_voxels(m, n, 0, N, seed=0)
@@ -51,6 +52,7 @@ def test_fullsize_sampled_parity(dev, cfg_name):
     gpu = tuple(t.index_select(0, sel).cpu().numpy() for t in (lam, x, it, cv))
     rep = PR.solve_parity(ent[idx], st, m, n, c["alpha"], c["tol"], c["maxit"], gpu)
     print(cfg_name, {kk: v for kk, v in rep.items() if kk != "details"})
+    PR.record(f"test_fullsize_sampled_parity[{cfg_name}]", dict(rep, tensors=N, sampled_tensors=int(len(idx))))
     assert rep["flag_unexplained"] == 0, rep
     assert rep["lam_unexplained"] == 0, rep
     assert rep["angle_unexplained"] == 0, rep
@@ -78,6 +80,7 @@ def test_blocked_default_sampled_parity(dev, m, n, N, alpha, k):
     gpu = tuple(t.index_select(0, sel).cpu().numpy() for t in (lam, x, it, cv))
     rep = PR.solve_parity(ent[idx], st, m, n, alpha, 1e-6, 100, gpu)
     print((m, n), {kk: v for kk, v in rep.items() if kk != "details"})
+    PR.record(f"test_blocked_default_sampled_parity[{m}-{n}]", dict(rep, tensors=N, sampled_tensors=int(len(idx))))
     assert rep["flag_unexplained"] == 0, rep
     assert rep["lam_unexplained"] == 0, rep
     assert rep["angle_unexplained"] == 0, rep

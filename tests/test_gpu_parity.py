@@ -410,6 +410,23 @@ def test_schedule7_bitwise(dev, m, n, V, S, alpha, maxit):
         assert np.array_equal(u, v)
 
 
+@pytest.mark.parametrize("alpha", ["per_tensor", "auto_max", 0.5, -0.5])
+@pytest.mark.parametrize("schedule", [6, 7])
+def test_schedules_6_7_shift_modes_bitwise(dev, alpha, schedule):
+    """Schedules 6 (predicated refill) and 7 (warp-tensor pipeline) with every shift kind (per-tensor, automatic,
+    positive, negative): bitwise equal to schedule 1."""
+    m, n, V, S = 4, 3, 700, 100
+    ent = syn.gen_voxels(m, n, 11, V, 3)
+    st = syn.gen_starts(S, n, 2)
+    if alpha == "per_tensor":
+        rng = np.random.default_rng(5)
+        alpha = torch.from_numpy(rng.choice([0.0, 0.5, -0.5, 1.0], size=V).astype(np.float32)).to(dev)
+    a = _solve(dev, m, n, ent, st, alpha, 1e-6, 200, schedule=1)
+    b = _solve(dev, m, n, ent, st, alpha, 1e-6, 200, schedule=schedule)
+    for u, v in zip(a, b):
+        assert np.array_equal(u, v)
+
+
 def test_records_only_overflow(dev):
     """Records-only path with tensors of more than 32 clusters (tight tolerances on unstructured odd-m tensors):
     those tensors take the raw-output + list-kernel route; records equal the two-pass form."""
