@@ -123,6 +123,9 @@ struct S43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 4)
 // form 2: the round-1 layout, x held as (x0, x1), (x2, x1) (slot 3 duplicates x1), monomials as 8 FMUL2
 template <int M, int N>
 struct X21 { static constexpr bool v = (M == 4 && N == 3 && (SSHOPM_43_FORM == 2 || SSHOPM_43_FORM == 3)); };
+#ifndef SSHOPM_X21_TAIL
+#define SSHOPM_X21_TAIL 1   // 1 (default): forms 2/3 with lambda, ||xhat||^2 and the update in scalar FP32 (C2 4.26 -> 4.22 ms)
+#endif
 template <int M, int N>
 __host__ __device__ constexpr int xslot(int i) {
   return X02<M, N>::v ? (i == 0 ? 0 : (i == 1 ? 2 : 1)) : i;
@@ -413,7 +416,34 @@ __device__ __forceinline__ float eval43(const Coefs<4, 3>& cf, const float2 (&xs
   return fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
 }
 
-#if SSHOPM_43_FORM == 2 && !defined(SSHOPM_SCALAR_MONO)
+#ifndef SSHOPM_MONO_MIX
+#define SSHOPM_MONO_MIX 0   // form 2 monomials: 0 = 8 FMUL2; 1 = 3 FMUL2 (degree 2) + 10 FMUL; 2 = 6 FMUL + 5 FMUL2
+#endif
+#if SSHOPM_43_FORM == 2 && !defined(SSHOPM_SCALAR_MONO) && SSHOPM_MONO_MIX == 1
+template <>
+__device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
+  const float2 x01 = xs[0], x21 = xs[1];
+  const float x0 = x01.x, x1 = x01.y, x2 = x21.x;
+  const float2 s0 = __fmul2_rn(bc(x0), x01);      // (x0x0, x0x1)
+  const float2 s1 = __fmul2_rn(x01, x21);         // (x0x2, x1x1)
+  const float2 s2 = __fmul2_rn(bc(x2), x21);      // (x2x2, x2x1)
+  mq[0] = x0 * s0.x; mq[1] = x0 * s0.y; mq[2] = x0 * s1.x; mq[3] = x0 * s1.y; mq[4] = x0 * s2.y;
+  mq[5] = x0 * s2.x; mq[6] = x1 * s1.y; mq[7] = x2 * s1.y; mq[8] = x1 * s2.x; mq[9] = x2 * s2.x;
+}
+#elif SSHOPM_43_FORM == 2 && !defined(SSHOPM_SCALAR_MONO) && SSHOPM_MONO_MIX == 2
+template <>
+__device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
+  const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
+  const float2 d0 = f2(x0 * x0, x0 * x1), d1 = f2(x0 * x2, x1 * x1), d2 = f2(x1 * x2, x2 * x2);
+  const float2 m01 = __fmul2_rn(bc(x0), d0);      // 000 001
+  const float2 m23 = __fmul2_rn(bc(x0), d1);      // 002 011
+  const float2 m45 = __fmul2_rn(bc(x0), d2);      // 012 022
+  const float2 m67 = __fmul2_rn(bc(x1), f2(d1.y, d2.x));   // 111 112
+  const float2 m89 = __fmul2_rn(bc(x2), d2);      // 122 222
+  mq[0] = m01.x; mq[1] = m01.y; mq[2] = m23.x; mq[3] = m23.y; mq[4] = m45.x;
+  mq[5] = m45.y; mq[6] = m67.x; mq[7] = m67.y; mq[8] = m89.x; mq[9] = m89.y;
+}
+#elif SSHOPM_43_FORM == 2 && !defined(SSHOPM_SCALAR_MONO)
 template <>
 __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&mq)[10]) {
   const float2 x01 = xs[0], x21 = xs[1];
@@ -591,6 +621,36 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
     if (!stop) {
       xs[0] = __fmul2_rn(h01, bc(r));
       xs[1].x = h2 * r;
+      lamp = lam;
+      ++k;
+    }
+    return;
+  } else if constexpr (X21<M, N>::v && SSHOPM_X21_TAIL == 1) {
+    // form-2 monomials and contraction; lambda, ||xhat||^2 and the update as scalar FP32 (no packed op
+    // next to the scalar ones there: DESIGN.md "pipe mix")
+    float mq[S::Q];
+    monomials<M, N>(xs, mq);
+    float2 gp[1];
+    float g2 = 0.f;
+    cf.contract(mq, gp, g2);
+    const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
+    const float g0 = gp[0].x, g1 = gp[0].y;
+    lam = fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
+    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
+    float h0, h1, h2;
+    if constexpr (SHIFT == 0) { h0 = g0; h1 = g1; h2 = g2; }
+    else if constexpr (SHIFT == 1) { h0 = fmaf(alpha, x0, g0); h1 = fmaf(alpha, x1, g1); h2 = fmaf(alpha, x2, g2); }
+    else if constexpr (SHIFT == 2) { h0 = fmaf(alpha, x0, -g0); h1 = fmaf(alpha, x1, -g1); h2 = fmaf(alpha, x2, -g2); }
+    else { h0 = fmaf(la, x0, g0 * ls); h1 = fmaf(la, x1, g1 * ls); h2 = fmaf(la, x2, g2 * ls); }
+    const float nn = fmaf(h2, h2, fmaf(h1, h1, h0 * h0));
+    const bool deg = !(nn >= 1.17549435e-38f);
+    if constexpr (KIDLE) stop = conv | (k >= maxit) | deg;
+    else stop = (!has) | conv | (k >= maxit) | deg;
+    const float r = rsqrt_ftz(nn);
+    if (!stop) {
+      const float y1 = h1 * r;
+      xs[0] = f2(h0 * r, y1);
+      xs[1] = f2(h2 * r, y1);
       lamp = lam;
       ++k;
     }
