@@ -55,7 +55,10 @@ size_t handle_workspace_bytes(const sshopm_ctx* h, int64_t N, int S) {
   return h->L ? workspace_bytes(h->L, N, S) : 256;          // the general kernel needs no workspace
 }
 
-int chunk_tensors_for(int S) { return (S >= 256) ? 1 : (256 + S - 1) / S; }
+#ifndef SSHOPM_CHUNK_ITEMS
+#define SSHOPM_CHUNK_ITEMS 256   // schedule 1: items per claimed chunk (whole tensors, at least one)
+#endif
+int chunk_tensors_for(int S) { return (S >= SSHOPM_CHUNK_ITEMS) ? 1 : (SSHOPM_CHUNK_ITEMS + S - 1) / S; }
 
 static size_t packed_region(const Launchers* L, int64_t N) { return ((size_t)N * (size_t)L->PW * 4 + 255) / 256 * 256; }
 

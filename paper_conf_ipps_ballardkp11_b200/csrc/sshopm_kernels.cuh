@@ -72,12 +72,14 @@ constexpr int round4(int v) { return (v + 3) / 4 * 4; }
 // branch over more arithmetic but let stopped lanes idle longer; measured on
 // B200 (C2, (4,3)): 1 step 4.90 ms, 2 steps 4.60, 3 steps 4.45, 4 steps 4.58
 // (best refill threshold each).  Shapes with costlier steps keep 2.
+// Round 2, (4,3) with the scalar-tail step: 4 steps per trip (C2 4.14 ms at K = 10; 3 steps 4.22 at K = 8,
+// 5 steps 4.34, 6 steps 4.34: profiles/r2/solve_variants_s6.jsonl).
 template <int M, int N>
 constexpr int steps_per_trip() {
 #ifdef SSHOPM_STEPS
   return SSHOPM_STEPS;
 #else
-  return (binom(M + N - 2, M - 1) * N <= 30) ? 3 : 2;
+  return (M == 4 && N == 3) ? 4 : ((binom(M + N - 2, M - 1) * N <= 30) ? 3 : 2);
 #endif
 }
 
@@ -914,7 +916,10 @@ sshopm_solve_kernel(const SolveParams p) {
         item = v0 * (Idx)S_ + (Idx)t;
         Idx tv;                                            // tensor of the item
         uint32_t s;                                        // its start
-        if (p.s_log2 >= 0) {                               // S a power of two (the paper's 128): shift and mask
+#ifndef SSHOPM_ASSUME_POW2
+#define SSHOPM_ASSUME_POW2 0   // experiment: compile only the power-of-two index path
+#endif
+        if (SSHOPM_ASSUME_POW2 || p.s_log2 >= 0) {         // S a power of two (the paper's 128): shift and mask
           tv = item >> p.s_log2;
           s = (uint32_t)item & p.s_mask;
         } else {
