@@ -41,17 +41,20 @@ def run_one(args):
         times = []
         for rep in range(args.reps + 2):
             flush.zero_()
-            tot.zero_()
+            if rep == 0 or not args.no_total:
+                tot.zero_()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
+            count = rep == 0 or not args.no_total       # --no-total: time without the iteration counter
             out = solver.solve(ent, st, alpha=cfg["alpha"], tol=cfg["tol"], maxit=cfg["maxit"], out=out,
-                               refill_threshold=k, schedule=sched, chunk_tensors=chunk, total_iters=tot)
+                               refill_threshold=k, schedule=sched, chunk_tensors=chunk,
+                               total_iters=tot if count else None)
             e1.record()
             torch.cuda.synchronize()
             if rep >= 2:
                 times.append(e0.elapsed_time(e1))
         ms = float(np.median(times))
-        its = int(tot.item())
+        its = int(tot.item())                            # from rep 0 (every rep when counting)
         F = solver.exec_flops_per_iter
         if cfg["alpha"] == 0.0:
             F -= 2 * n                       # alpha = 0: no shift FMAs (bench.py's count)
@@ -75,12 +78,13 @@ def main():
     ap.add_argument("--sets", default="1:0:0")
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--libs", default="")
+    ap.add_argument("--no-total", action="store_true")
     a = ap.parse_args()
     if a.libs and "SSHOPM_LIBRARY" not in os.environ:
         for lib in a.libs.split(","):
             env = dict(os.environ, SSHOPM_LIBRARY=os.path.abspath(lib))
             cmd = [sys.executable, __file__, "--config", a.config, "--voxels", str(a.voxels), "--sets", a.sets,
-                   "--reps", str(a.reps)]
+                   "--reps", str(a.reps)] + (["--no-total"] if a.no_total else [])
             subprocess.run(cmd, env=env, check=False)
         return
     run_one(a)
