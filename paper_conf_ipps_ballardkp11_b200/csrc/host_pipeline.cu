@@ -11,7 +11,10 @@
 // one handle serialise on the cache mutex.  sshopm_destroy frees the cache.
 #include <cstdlib>
 #include <cstring>
+#include <chrono>
 #include <mutex>
+#include <vector>
+#include <cstdio>
 
 #include "api_internal.h"
 #include "sshopm.h"
@@ -73,6 +76,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
                                int32_t* h_out_count, float* h_out_lambda, float* h_out_x, int32_t* h_out_mult,
                                int32_t* h_out_rep, float* h_raw_lambda, float* h_raw_x, int32_t* h_raw_iters,
                                uint8_t* h_raw_converged, int64_t chunk_tensors, unsigned long long* h_total_iters) {
+  const auto t_enter = std::chrono::steady_clock::now();
   if (!h || N < 0 || S < 1 || maxit < 0 || kmax < 1) return SSHOPM_EINVAL;
   if (h_total_iters) *h_total_iters = 0;
   if (N == 0) return SSHOPM_OK;
@@ -97,6 +101,11 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   std::lock_guard<std::mutex> lock(c->mu);
   int dev = 0;
   cudaGetDevice(&dev);
+  // SSHOPM_E2E_TRACE=file: append a per-chunk timeline (H2D start/end, kernels end, D2H end; ms from the
+  // first event) to `file` — a diagnostic for the pipeline's exposed fill / drain, off by default
+  static const char* trace_path = getenv("SSHOPM_E2E_TRACE");
+  std::vector<cudaEvent_t> tev;
+  std::vector<long long> tcn;
   int rc = SSHOPM_OK;
   cudaError_t e = cudaSuccess;
 #define CK(call, where) do { e = (call); if (e != cudaSuccess) { rc = (e == cudaErrorMemoryAllocation) ? SSHOPM_ENOMEM : cuda_fail(e, where); goto done; } } while (0)
@@ -134,6 +143,8 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   CK(cudaMemcpyAsync(c->d_starts, h_starts, sizeof(float) * S * n, cudaMemcpyHostToDevice, c->slots[0].st), "run_host: H2D");
   CK(cudaMemsetAsync(c->d_total, 0, sizeof(unsigned long long), c->slots[0].st), "run_host: memset");
   CK(cudaStreamSynchronize(c->slots[0].st), "run_host: sync");
+  {
+  const auto t_setup = std::chrono::steady_clock::now();
   for (long long c0 = 0, ci = 0, cn = 0; c0 < N; c0 += cn, ++ci) {
     Slot& s = c->slots[ci % kSlots];
     // ramped chunk sizes: chunk/4, chunk/2 first and last, so the exposed pipeline fill (first H2D) and
@@ -149,7 +160,17 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     }
     if (cn < 1) cn = 1;
     if (cn > left) cn = left;
+    auto mark = [&]() {
+      if (!trace_path) return;
+      cudaEvent_t ev;
+      cudaEventCreate(&ev);
+      cudaEventRecord(ev, s.st);
+      tev.push_back(ev);
+    };
+    if (trace_path) tcn.push_back(cn);
+    mark();
     CK(cudaMemcpyAsync(s.ent, h_entries + c0 * U, sizeof(float) * cn * U, cudaMemcpyHostToDevice, s.st), "run_host: H2D");
+    mark();
     sshopm_solve_opts o;
     memset(&o, 0, sizeof(o));
     o.d_total_iters = c->d_total;
@@ -158,6 +179,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     rc = sshopm_solve_dedup(h, cn, s.ent, S, c->d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, lam_tol, ang_tol,
                             kmax, s.cnt, s.olam, s.ox, s.mult, s.rep, &o, s.st);
     if (rc != SSHOPM_OK) goto done;
+    mark();
     CK(cudaMemcpyAsync(h_out_count + c0, s.cnt, sizeof(int32_t) * cn, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     CK(cudaMemcpyAsync(h_out_lambda + c0 * kmax, s.olam, sizeof(float) * cn * kmax, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     CK(cudaMemcpyAsync(h_out_x + c0 * kmax * n, s.ox, sizeof(float) * cn * kmax * n, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
@@ -170,9 +192,28 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
       CK(cudaMemcpyAsync(h_raw_iters + c0 * S, s.it, sizeof(int32_t) * cn * S, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
       CK(cudaMemcpyAsync(h_raw_converged + c0 * S, s.cv, cn * S, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     }
+    mark();
   }
+  const auto t_enq = std::chrono::steady_clock::now();
   for (int i = 0; i < kSlots; ++i)
     if (c->slots[i].st) CK(cudaStreamSynchronize(c->slots[i].st), "run_host: sync");
+  if (trace_path && !tev.empty()) {
+    const auto t_sync = std::chrono::steady_clock::now();
+    auto ms = [](std::chrono::steady_clock::duration d) { return std::chrono::duration<double, std::milli>(d).count(); };
+    if (FILE* f = fopen(trace_path, "a")) {
+      fprintf(f, "# run_host N=%lld chunk=%lld: host ms setup %.4f, enqueue %.4f, sync %.4f\n", (long long)N, chunk,
+              ms(t_setup - t_enter), ms(t_enq - t_setup), ms(t_sync - t_enq));
+      fprintf(f, "# chunk tensors h2d_start h2d_end kernels_end d2h_end (ms)\n");
+      for (size_t i = 0; i + 3 < tev.size(); i += 4) {
+        float t[4];
+        for (int j = 0; j < 4; ++j) cudaEventElapsedTime(&t[j], tev[0], tev[i + j]);
+        fprintf(f, "%zu %lld %.4f %.4f %.4f %.4f\n", i / 4, tcn[i / 4], t[0], t[1], t[2], t[3]);
+      }
+      fclose(f);
+    }
+    for (cudaEvent_t ev : tev) cudaEventDestroy(ev);
+  }
+  }
   if (h_total_iters) CK(cudaMemcpy(h_total_iters, c->d_total, sizeof(unsigned long long), cudaMemcpyDeviceToHost), "run_host: D2H");
 #undef CK
 done:

@@ -109,7 +109,59 @@ def pool_policy(ev, STEPS, nwarps=8):
     return useful / (64 * steps)
 
 
-if __name__ == "__main__":
+def affinity_policy(ev, K, STEPS, nwarps=8):
+    """Two slots per lane, the lane owns one tensor at a time: when >= K of the warp's 64 slots are stopped,
+    every stopped slot takes its lane's tensor's next start; a lane whose tensor has no start left and whose
+    two slots are both stopped claims the next tensor (coefficient reload).  Returns (utilisation, refill
+    events per useful slot-step, tensor switches per useful slot-step)."""
+    T, S = ev.shape
+    per = T // nwarps
+    steps = useful = refills = switches = 0
+    for w in range(nwarps):
+        nxt_t = w * per
+        end_t = (w + 1) * per
+        ten = np.full(32, -1)
+        pos = np.full(32, S)
+        rem = np.zeros((32, 2), np.int64)
+        while True:
+            stopped = rem == 0
+            cnt = int(stopped.sum())
+            live = (pos < S).any() or nxt_t < end_t
+            if (cnt >= K or not live) and cnt:
+                refills += 1
+                for l in range(32):
+                    if pos[l] >= S and stopped[l].all() and nxt_t < end_t:
+                        ten[l], pos[l] = nxt_t, 0
+                        nxt_t += 1
+                        switches += 1
+                    for sl in range(2):
+                        if rem[l, sl] == 0 and pos[l] < S:
+                            rem[l, sl] = ev[ten[l], pos[l]]
+                            pos[l] += 1
+                if not live and rem.sum() == 0:
+                    break
+            for _ in range(STEPS):
+                a = rem > 0
+                useful += int(a.sum())
+                rem[a] -= 1
+                steps += 1
+    return useful / (64 * steps), refills / useful, switches / useful
+
+
+def main_affinity():
+    ev = iteration_counts(int(sys.argv[2]) if len(sys.argv) > 2 else 1024)
+    for K, ST in [(8, 2), (12, 2), (16, 2), (12, 3), (16, 3), (20, 3), (24, 4), (16, 4)]:
+        u, r, s = affinity_policy(ev, K, ST)
+        print(f"affinity K={K} STEPS={ST}: slot utilisation {u:.3f}, refill events per useful slot-step {r:.4f}, "
+              f"tensor switches per useful slot-step {s:.5f}")
+    for K, ST in [(10, 4), (8, 3)]:
+        u, e = item_policy(ev, K, ST)
+        print(f"item  K={K} STEPS={ST}: lane utilisation {u:.3f}")
+
+
+if __name__ == "__main__" and sys.argv[1:2] == ["affinity"]:
+    main_affinity()
+elif __name__ == "__main__":
     ev = iteration_counts(int(sys.argv[1]) if len(sys.argv) > 1 else 1024)
     print(f"mean evaluations per item {ev.mean():.2f}, p99 {np.percentile(ev, 99):.0f}")
     for K, ST in [(8, 3), (6, 3), (4, 3), (4, 1)]:
