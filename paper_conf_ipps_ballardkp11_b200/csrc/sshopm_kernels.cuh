@@ -125,6 +125,10 @@ struct S43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 4)
 // form 2: the round-1 layout, x held as (x0, x1), (x2, x1) (slot 3 duplicates x1), monomials as 8 FMUL2
 template <int M, int N>
 struct X21 { static constexpr bool v = (M == 4 && N == 3 && (SSHOPM_43_FORM == 2 || SSHOPM_43_FORM == 3)); };
+#ifndef SSHOPM_GEN_TAIL
+#define SSHOPM_GEN_TAIL 1   // other n = 3 shapes with rows of <= 64 words: scalar lambda / ||xhat||^2 / update
+                            // (C3 (6,3) solve 11.85 -> 11.60 ms; (8,3) is 0.9% slower with it, so excluded)
+#endif
 #ifndef SSHOPM_X21_TAIL
 #define SSHOPM_X21_TAIL 1   // 1 (default): forms 2/3 with lambda, ||xhat||^2 and the update in scalar FP32 (C2 4.26 -> 4.22 ms)
 #endif
@@ -653,6 +657,34 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
       const float y1 = h1 * r;
       xs[0] = f2(h0 * r, y1);
       xs[1] = f2(h2 * r, y1);
+      lamp = lam;
+      ++k;
+    }
+    return;
+  } else if constexpr (N == 3 && SSHOPM_GEN_TAIL == 1 && S::Q * N <= 64) {
+    // other n = 3 shapes: the library contraction, then lambda, ||xhat||^2 and the update in scalar FP32
+    float mq[S::Q];
+    monomials<M, N>(xs, mq);
+    float2 gp[1];
+    float g2 = 0.f;
+    cf.contract(mq, gp, g2);
+    const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
+    const float g0 = gp[0].x, g1 = gp[0].y;
+    lam = fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
+    conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
+    float h0, h1, h2;
+    if constexpr (SHIFT == 0) { h0 = g0; h1 = g1; h2 = g2; }
+    else if constexpr (SHIFT == 1) { h0 = fmaf(alpha, x0, g0); h1 = fmaf(alpha, x1, g1); h2 = fmaf(alpha, x2, g2); }
+    else if constexpr (SHIFT == 2) { h0 = fmaf(alpha, x0, -g0); h1 = fmaf(alpha, x1, -g1); h2 = fmaf(alpha, x2, -g2); }
+    else { h0 = fmaf(la, x0, g0 * ls); h1 = fmaf(la, x1, g1 * ls); h2 = fmaf(la, x2, g2 * ls); }
+    const float nn = fmaf(h2, h2, fmaf(h1, h1, h0 * h0));
+    const bool deg = !(nn >= 1.17549435e-38f);
+    if constexpr (KIDLE) stop = conv | (k >= maxit) | deg;
+    else stop = (!has) | conv | (k >= maxit) | deg;
+    const float r = rsqrt_ftz(nn);
+    if (!stop) {
+      xs[0] = f2(h0 * r, h1 * r);
+      xs[1].x = h2 * r;
       lamp = lam;
       ++k;
     }
