@@ -124,7 +124,10 @@ template <int M, int N>
 struct S43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 4); };
 // form 2: the round-1 layout, x held as (x0, x1), (x2, x1) (slot 3 duplicates x1), monomials as 8 FMUL2
 template <int M, int N>
-struct X21 { static constexpr bool v = (M == 4 && N == 3 && (SSHOPM_43_FORM == 2 || SSHOPM_43_FORM == 3)); };
+struct X21 { static constexpr bool v = (M == 4 && N == 3 && (SSHOPM_43_FORM == 2 || SSHOPM_43_FORM == 3 || SSHOPM_43_FORM == 5)); };
+// form 5: the form-2 layout, g by Horner in x0 over shared (x1, x2) monomials, (g0, g1) as FFMA2, g2 scalar
+template <int M, int N>
+struct H43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 5); };
 #ifndef SSHOPM_GEN_TAIL
 #define SSHOPM_GEN_TAIL 1   // other n = 3 shapes with rows of <= 64 words: scalar lambda / ||xhat||^2 / update
                             // (C3 (6,3) solve 11.85 -> 11.60 ms; (8,3) is 0.9% slower with it, so excluded)
@@ -483,6 +486,47 @@ __device__ __forceinline__ void monomials<4, 3>(const float2 (&xs)[2], float (&m
 }
 #endif
 
+// (4,3), form 5: Eq. 6 regrouped as a polynomial in x0 whose coefficients are forms in (x1, x2),
+//   g_j = x0 (x0 (x0 B_000j + B_001j x1 + B_002j x2) + Q_j) + C_j,
+//   Q_j = B_011j x1^2 + B_012j x1x2 + B_022j x2^2,  C_j = B_111j x1^3 + B_112j x1^2x2 + B_122j x1x2^2 + B_222j x2^3
+// (B_qj = B-form word of monomial q for output j): 36 multiply-adds per step plus 7 shared products
+// (43 FP32 pipe operations instead of 30 + 16); (g0, g1) run as FFMA2 on the B-form word pairs with
+// the shared value broadcast, g2 as scalar FFMA.  State layout of form 2: xs = (x0, x1), (x2, x1).
+__device__ __forceinline__ void horner43(const Coefs<4, 3>& cf, const float2 (&xs)[2], float& g0, float& g1, float& g2) {
+  const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
+  const float2 p21 = xs[1];                          // (x2, x1)
+  const float2 s = __fmul2_rn(bc(x1), p21);          // (x1x2, x1x1)
+  const float s22 = x2 * x2;
+  const float2 c1 = __fmul2_rn(bc(s.y), p21);        // (x1^2 x2, x1^3)
+  const float2 c2 = __fmul2_rn(bc(s22), p21);        // (x2^3, x1 x2^2)
+  float2 L = __fmul2_rn(cf.template pair<2>(), bc(x1));
+  L = __ffma2_rn(cf.template pair<4>(), bc(x2), L);
+  float2 t = __ffma2_rn(cf.template pair<0>(), bc(x0), L);
+  float2 Q = __fmul2_rn(cf.template pair<6>(), bc(s.y));
+  Q = __ffma2_rn(cf.template pair<8>(), bc(s.x), Q);
+  Q = __ffma2_rn(cf.template pair<10>(), bc(s22), Q);
+  t = __ffma2_rn(t, bc(x0), Q);
+  float2 C = __fmul2_rn(cf.template pair<12>(), bc(c1.y));
+  C = __ffma2_rn(cf.template pair<14>(), bc(c1.x), C);
+  C = __ffma2_rn(cf.template pair<16>(), bc(c2.y), C);
+  C = __ffma2_rn(cf.template pair<18>(), bc(c2.x), C);
+  const float2 g01 = __ffma2_rn(t, bc(x0), C);
+  g0 = g01.x;
+  g1 = g01.y;
+  float L2 = cf.template word<21>() * x1;
+  L2 = fmaf(cf.template word<22>(), x2, L2);
+  float t2 = fmaf(cf.template word<20>(), x0, L2);
+  float Q2 = cf.template word<23>() * s.y;
+  Q2 = fmaf(cf.template word<24>(), s.x, Q2);
+  Q2 = fmaf(cf.template word<25>(), s22, Q2);
+  t2 = fmaf(t2, x0, Q2);
+  float C2 = cf.template word<26>() * c1.y;
+  C2 = fmaf(cf.template word<27>(), c1.x, C2);
+  C2 = fmaf(cf.template word<28>(), c2.y, C2);
+  C2 = fmaf(cf.template word<29>(), c2.x, C2);
+  g2 = fmaf(t2, x0, C2);
+}
+
 // (4,3), form 4: all-scalar evaluation (16 FMUL monomials, 30 FFMA, lambda as an FMA chain).
 __device__ __forceinline__ float eval43s(const Coefs<4, 3>& cf, float x0, float x1, float x2, float& g0, float& g1,
                                          float& g2) {
@@ -632,15 +676,21 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
     }
     return;
   } else if constexpr (X21<M, N>::v && SSHOPM_X21_TAIL == 1) {
-    // form-2 monomials and contraction; lambda, ||xhat||^2 and the update as scalar FP32 (no packed op
-    // next to the scalar ones there: DESIGN.md "pipe mix")
-    float mq[S::Q];
-    monomials<M, N>(xs, mq);
-    float2 gp[1];
-    float g2 = 0.f;
-    cf.contract(mq, gp, g2);
+    // form-2 monomials and contraction (form 5: Horner in x0); lambda, ||xhat||^2 and the update as scalar
+    // FP32 (no packed op next to the scalar ones there: DESIGN.md "pipe mix")
+    float g0, g1, g2;
+    if constexpr (H43<M, N>::v) {
+      horner43(cf, xs, g0, g1, g2);
+    } else {
+      float mq[S::Q];
+      monomials<M, N>(xs, mq);
+      float2 gp[1];
+      g2 = 0.f;
+      cf.contract(mq, gp, g2);
+      g0 = gp[0].x;
+      g1 = gp[0].y;
+    }
     const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
-    const float g0 = gp[0].x, g1 = gp[0].y;
     lam = fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
     conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
     float h0, h1, h2;
@@ -884,6 +934,9 @@ sshopm_solve_kernel(const SolveParams p) {
   int k = 0;
   bool has = false, stop = true, conv = false;
   Idx item = 0;
+#ifdef SSHOPM_SKIP_RELOAD
+  Idx cur_tv = (Idx)-1;
+#endif
   float la = 0.f, ls = 1.f;  // SHIFT == 3: per-lane |alpha| and sign: xhat = ls*g + la*x
   uint32_t it_sum = 0;       // per-lane sum of iterations (<= items per lane x maxit; flushed as 64-bit)
   // refill threshold: K idle lanes while items remain, all 32 once the chunks are exhausted,
@@ -965,7 +1018,11 @@ sshopm_solve_kernel(const SolveParams p) {
           ls = at >= 0.f ? 1.f : -1.f;                     // Fig. 1 lines 2-5 (R5: alpha = 0 -> "+")
           la = fabsf(at);
         }
+#ifdef SSHOPM_SKIP_RELOAD
+        if (tv != cur_tv) { cf.load(p.packed + tv * (Idx)(S::PW / 4)); cur_tv = tv; }   // experiment: same tensor -> keep the rows
+#else
         cf.load(p.packed + tv * (Idx)(S::PW / 4));
+#endif
         float v[4 * SST4];
 #pragma unroll
         for (int i = 0; i < SST4; ++i) {
@@ -1466,7 +1523,14 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
     }
     if constexpr (X21<M, N>::v) xs[1].y = xs[0].y;
     float lam;
-    if constexpr (S43<M, N>::v) {
+    if constexpr (H43<M, N>::v) {
+      float g0, g1, g2;
+      horner43(cf, xs, g0, g1, g2);
+      lam = fmaf(xs[1].x, g2, fmaf(xs[0].y, g1, xs[0].x * g0));
+      out_g[i * N + 0] = g0;
+      out_g[i * N + 1] = g1;
+      out_g[i * N + 2] = g2;
+    } else if constexpr (S43<M, N>::v) {
       float g0, g1, g2;
       lam = eval43s(cf, xs[0].x, xs[0].y, xs[1].x, g0, g1, g2);
       out_g[i * N + 0] = g0;
