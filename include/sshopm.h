@@ -105,6 +105,9 @@ int sshopm_solve(sshopm_t h, int64_t N, const float* d_entries, int S, const flo
  * themselves (cudaMallocAsync / cudaFreeAsync on the stream). */
 int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes);
 
+/* Scratch bytes of the records path (fuse_dedup = 4): N * S * 16 * ceil((n + 1) / 4). */
+int sshopm_records_size(sshopm_t h, int64_t N, int S, size_t* bytes);
+
 /* Tuning / instrumentation knobs for sshopm_solve_ex (0 / NULL = library default). */
 typedef struct {
   int refill_threshold;            /* lanes that must be idle before a warp refills (1..32); default per (m, n) */
@@ -125,9 +128,15 @@ typedef struct {
                                       thread per start (the paper's mapping); 3-5 also force the
                                       table-driven path on compiled shapes (5 returns EUNSUPPORTED if its
                                       shared memory does not fit; the default then falls back to 3, then 4). */
-  int fuse_dedup;                  /* sshopm_solve_dedup only: 0 = default (two passes; fastest on B200),
+  int fuse_dedup;                  /* sshopm_solve_dedup only: 0 = default (two passes),
                                       1 = solve warps cluster their chunks, 3 = one dedup warp per CTA,
-                                      2 = records only (schedule 7 pipeline); results identical */
+                                      2 = records only (schedule 7 pipeline), 4 = records path (schedule 8):
+                                      lanes own units of consecutive starts of one tensor (no coefficient
+                                      reload per item), each start leaves one 16-byte (lambda | NaN, x)
+                                      record in scratch that the dedup reads; the raw per-start outputs are
+                                      not written (their pointers may be NULL) and out_iters is not
+                                      produced (d_total_iters still counts).  Dedup outputs identical in
+                                      every mode. */
   int alpha_mode;                  /* shift: 0 = the scalar alpha argument (default);
                                       1 = per tensor, d_alpha[N] (device); 2 = per tensor automatic convex shift
                                       alpha_t = +(m-1) sum_{all indices} |a| (>= beta(A): lambda_k nondecreasing,
@@ -136,6 +145,10 @@ typedef struct {
   const float* d_alpha;            /* alpha_mode 1: per-tensor shifts [N] */
   int chunk_tensors;               /* schedule 6: tensors per work chunk a warp claims (0 = default:
                                       up to 1024 items, at least 8 chunks per resident warp) */
+  void* d_records;                 /* fuse_dedup = 4: optional caller-owned scratch for the per-start records,
+                                      16-byte aligned, >= sshopm_records_size bytes (else allocated on the stream) */
+  size_t records_bytes;            /* its size */
+  int unit_starts;                 /* fuse_dedup = 4: starts per work unit a lane claims (0 = default 32) */
 } sshopm_solve_opts;
 
 /* sshopm_solve with options (opts may be NULL).  Launches two kernels on

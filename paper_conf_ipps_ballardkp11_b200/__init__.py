@@ -37,7 +37,8 @@ class _Opts(ctypes.Structure):
     _fields_ = [("refill_threshold", ctypes.c_int), ("ctas_per_sm", ctypes.c_int),
                 ("d_total_iters", ctypes.c_void_p), ("d_workspace", ctypes.c_void_p),
                 ("workspace_bytes", ctypes.c_size_t), ("schedule", ctypes.c_int), ("fuse_dedup", ctypes.c_int),
-                ("alpha_mode", ctypes.c_int), ("d_alpha", ctypes.c_void_p), ("chunk_tensors", ctypes.c_int)]
+                ("alpha_mode", ctypes.c_int), ("d_alpha", ctypes.c_void_p), ("chunk_tensors", ctypes.c_int),
+                ("d_records", ctypes.c_void_p), ("records_bytes", ctypes.c_size_t), ("unit_starts", ctypes.c_int)]
 
 ALPHA_MODES = {"scalar": 0, "per_tensor": 1, "auto_max": 2, "auto_min": 3}
 
@@ -67,6 +68,7 @@ def lib():
         "sshopm_run_host": (I, [P, I64, P, I, P, F, F, I, F, F, I, P, P, P, P, P, P, P, P, P, I64, P]),
         "sshopm_launch_count": (I, [P, ctypes.POINTER(I64)]),
         "sshopm_workspace_size": (I, [P, I64, I, ctypes.POINTER(ctypes.c_size_t)]),
+        "sshopm_records_size": (I, [P, I64, I, ctypes.POINTER(ctypes.c_size_t)]),
         "sshopm_status_string": (ctypes.c_char_p, [I]),
         "sshopm_last_cuda_error": (ctypes.c_char_p, []),
         "sshopm_supported_shapes": (ctypes.c_char_p, []),
@@ -224,6 +226,25 @@ class Solver:
         base = ws.data_ptr()
         return ctypes.c_void_p((base + 255) // 256 * 256), need
 
+    def _records(self, N, S, device, stream=None):
+        """Record scratch of the records path (fuse_dedup = 4), cached per (device, stream) like the workspace."""
+        b = ctypes.c_size_t()
+        _check(lib().sshopm_records_size(self._h, int(N), int(S), ctypes.byref(b)), "sshopm_records_size")
+        need = int(b.value)
+        torch = _torch()
+        st = torch.cuda.current_stream(device) if stream is None else stream
+        key = ("rec", str(device), int(st.cuda_stream))
+        buf = self._ws.get(key)
+        if buf is None or buf.numel() < need:
+            with torch.cuda.stream(st):
+                buf = torch.empty(need + 256, dtype=torch.uint8, device=device)
+            old = self._ws.get(key)
+            if old is not None:
+                old.record_stream(st)
+            self._ws[key] = buf
+        base = buf.data_ptr()
+        return ctypes.c_void_p((base + 255) // 256 * 256), need
+
     @staticmethod
     def _alpha_opts(alpha, N, opts):
         """alpha: float (scalar shift), a CUDA float32 tensor [N] (per tensor), or 'auto_max' / 'auto_min'."""
@@ -296,16 +317,42 @@ class Solver:
 
     def solve_dedup(self, entries, starts, alpha=0.0, tol=1e-6, maxit=100, lam_tol=1e-2, ang_tol=0.05, kmax=8,
                     out=None, dedup_out=None, refill_threshold=0, ctas_per_sm=0, total_iters=None, stream=None,
-                    schedule=0, fused=False, records_only=False, warp_specialized=False):
+                    schedule=0, fused=False, records_only=False, warp_specialized=False, records=False,
+                    unit_starts=0):
         """Fused solve + dedup (sshopm_solve_dedup).  Returns (raw outputs, dedup outputs) as in solve() / dedup().
         fused: cluster inside the solve kernel (schedule 1 ring, or schedule 7 staging).  records_only: the
         schedule-7 pipeline clusters in-kernel and leaves the raw outputs unwritten (they are scratch).
-        warp_specialized: one warp per CTA of the solve kernel clusters the chunks the other seven complete."""
+        warp_specialized: one warp per CTA of the solve kernel clusters the chunks the other seven complete.
+        records: the records path (schedule 8, fuse_dedup = 4): lanes own units of `unit_starts` starts of one
+        tensor, per-start results go to a 16-byte record scratch the dedup reads; no raw outputs (returns
+        (None, dedup outputs))."""
         torch = _torch()
         N, S = int(entries.shape[0]), int(starts.shape[0])
         pe = _dev(entries, torch.float32, (N, self.U), "entries")
         ps = _dev(starts, torch.float32, (S, self.n), "starts")
         dev = entries.device
+        if records:
+            if dedup_out is None:
+                dedup_out = (torch.empty((N,), dtype=torch.int32, device=dev),
+                             torch.empty((N, kmax), dtype=torch.float32, device=dev),
+                             torch.empty((N, kmax, self.n), dtype=torch.float32, device=dev),
+                             torch.empty((N, kmax), dtype=torch.int32, device=dev),
+                             torch.empty((N, kmax), dtype=torch.int32, device=dev))
+            c, ol, ox, om, orp = dedup_out
+            dargs = (_dev(c, torch.int32, (N,), "out_count"), _dev(ol, torch.float32, (N, kmax), "out_clambda"),
+                     _dev(ox, torch.float32, (N, kmax, self.n), "out_cx"), _dev(om, torch.int32, (N, kmax), "out_mult"),
+                     _dev(orp, torch.int32, (N, kmax), "out_rep"))
+            wsp, wsb = self._workspace(N, S, dev, stream) if N > 0 else (None, 0)
+            rp, rb = self._records(N, S, dev, stream) if N > 0 else (None, 0)
+            opts = _Opts(int(refill_threshold), int(ctas_per_sm), None, wsp, wsb, int(schedule), 4)
+            opts.d_records, opts.records_bytes, opts.unit_starts = rp, rb, int(unit_starts)
+            alpha = self._alpha_opts(alpha, N, opts)
+            if total_iters is not None:
+                opts.d_total_iters = total_iters.data_ptr()
+            _check(lib().sshopm_solve_dedup(self._h, N, pe, S, ps, float(alpha), float(tol), int(maxit), None, None,
+                                            None, None, float(lam_tol), float(ang_tol), int(kmax), *dargs,
+                                            ctypes.byref(opts), _stream(stream)), "sshopm_solve_dedup")
+            return None, dedup_out
         if out is None:
             out = (torch.empty((N, S), dtype=torch.float32, device=dev),
                    torch.empty((N, S, self.n), dtype=torch.float32, device=dev),

@@ -24,6 +24,9 @@ struct Launchers {
                           const float* x, float ctol, int8_t* out, int grid, cudaStream_t st);
   cudaError_t (*apply)(long long n_items, const float4* packed, const float* x, float* g, float* lam, int grid,
                        cudaStream_t st);
+  // records path (schedule 8, sshopm_solve_dedup with fuse_dedup = 4)
+  cudaError_t (*occupancy_rec)(int shift, int* blocks_per_sm);
+  cudaError_t (*solve_rec)(const RecParams& p, int shift, int grid, cudaStream_t st);
 };
 
 }  // namespace sshopm

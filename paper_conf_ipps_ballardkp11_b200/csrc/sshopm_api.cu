@@ -261,17 +261,107 @@ int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes) {
   return SSHOPM_OK;
 }
 
+int sshopm_records_size(sshopm_t h, int64_t N, int S, size_t* bytes) {
+  if (!h || N < 0 || S < 0 || !bytes) return SSHOPM_EINVAL;
+  *bytes = (size_t)N * (size_t)S * 16u * (size_t)sshopm::dd_rec4(h->n);
+  return SSHOPM_OK;
+}
+
 }  // extern "C"
 
 namespace sshopm {
 // The solve (pack + solve kernels) and, if dd != null, the fused dedup (ring
 // in the solve kernel + sshopm_dedup_list_kernel for untracked chunks), or the
 // standalone dedup after the solve when the fused form does not apply.
+// Records path (fuse_dedup = 4, schedule 8): pack, sshopm_solve_rec_kernel into the per-start record scratch,
+// dedup of the records.  The raw per-start outputs are not written.
+static int solve_records(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts, float alpha,
+                         float tol, int maxit, const sshopm_solve_opts* opts, const DedupParams* dd, cudaStream_t st) {
+  const Launchers* L = h->L;
+  const int sms = device_sms();
+  if (sms <= 0) return cuda_fail(cudaGetLastError(), "sshopm_solve_dedup: no device");
+  const int alpha_mode = opts->alpha_mode;
+  if (alpha_mode < 0 || alpha_mode > 3) return SSHOPM_EINVAL;
+  if (alpha_mode == 1 && !opts->d_alpha) return SSHOPM_EINVAL;
+  const int shift = alpha_mode ? 3 : (alpha == 0.f ? 0 : (alpha > 0.f ? 1 : 2));
+  if (opts->unit_starts < 0) return SSHOPM_EINVAL;
+  int unit = opts->unit_starts > 0 ? opts->unit_starts : 32;
+  if (unit > S) unit = S;
+  const long long upt = (S + unit - 1) / unit;
+  const long long n_units = (long long)N * upt;
+  if (n_units >= (1LL << 32) - (1LL << 20) || (long long)N * S >= (1LL << 32) - 1) return SSHOPM_EUNSUPPORTED;
+  const size_t rbytes = (size_t)N * (size_t)S * 16u * (size_t)dd_rec4(h->n);
+  float4* rec = reinterpret_cast<float4*>(opts->d_records);
+  bool own = false;
+  if (rec) {
+    if (opts->records_bytes < rbytes || ((uintptr_t)rec & 15)) return SSHOPM_EINVAL;
+  } else {
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&rec), rbytes, st);
+    if (e == cudaErrorMemoryAllocation) return SSHOPM_ENOMEM;
+    if (e != cudaSuccess) return cuda_fail(e, "records: cudaMallocAsync");
+    own = true;
+  }
+  auto done = [&](int rc) {
+    if (own) {
+      cudaError_t e = cudaFreeAsync(rec, st);
+      if (rc == SSHOPM_OK && e != cudaSuccess) rc = cuda_fail(e, "records: cudaFreeAsync");
+    }
+    return rc;
+  };
+  int bps = 0;
+  cudaError_t e = L->occupancy_rec(shift, &bps);
+  if (e != cudaSuccess) return done(cuda_fail(e, "sshopm_solve_dedup: occupancy"));
+  if (bps < 1) bps = 1;
+  if (opts->ctas_per_sm > 0 && opts->ctas_per_sm < bps) bps = opts->ctas_per_sm;
+  long long grid = (long long)sms * bps;
+  if (grid * 256 > n_units) grid = (n_units + 255) / 256;          // a lane per unit at most
+  if (grid < 1) grid = 1;
+  Workspace ws;
+  int rc = acquire_workspace(L, N, S, opts->d_workspace, opts->workspace_bytes, st, &ws);
+  if (rc != SSHOPM_OK) return done(rc);
+  long long pgrid = ((N > S ? N : S) + 255) / 256;
+  if (pgrid > (long long)sms * 8) pgrid = (long long)sms * 8;
+  e = L->pack(N, d_entries, ws.packed, ws.counter, S, d_starts, ws.starts_n, alpha_mode,
+              alpha_mode == 1 ? opts->d_alpha : nullptr, ws.alpha_t, (int)pgrid, st);
+  if (e != cudaSuccess) { release_workspace(&ws, st); return done(cuda_fail(e, "sshopm_solve_dedup: pack launch")); }
+  RecParams p;   // counter: word 0 of the workspace header, zeroed by the pack kernel
+  p.packed = ws.packed;
+  p.starts_n = reinterpret_cast<const float4*>(ws.starts_n);
+  p.rec = rec;
+  p.total_iters = opts->d_total_iters;
+  p.counter = ws.counter;
+  p.n_units = (uint32_t)n_units;
+  p.units_per_tensor = (uint32_t)upt;
+  p.unit = (uint32_t)unit;
+  p.S = (uint32_t)S;
+  p.div_upt = make_fastdiv((uint32_t)upt);
+  p.alpha = alpha;
+  p.tol = tol;
+  p.alpha_t = ws.alpha_t;
+  p.maxit = maxit;
+  int k = opts->refill_threshold > 0 ? opts->refill_threshold : 4;
+  p.refill_k = k < 1 ? 1 : (k > 32 ? 32 : k);
+  e = L->solve_rec(p, shift, (int)grid, st);
+  if (e != cudaSuccess) { release_workspace(&ws, st); return done(cuda_fail(e, "sshopm_solve_dedup: launch")); }
+  h->launches.fetch_add(2);
+  DedupParams q = *dd;
+  q.rec = rec;
+  rc = launch_dedup(h->m, h->n, q, st);
+  if (rc == SSHOPM_OK) h->launches.fetch_add(1);
+  int r2 = release_workspace(&ws, st);
+  return done(rc != SSHOPM_OK ? rc : r2);
+}
+
 static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, const float* d_starts, float alpha,
                       float tol, int maxit, float* d_out_lambda, float* d_out_x, int32_t* d_out_iters,
                       uint8_t* d_out_converged, const sshopm_solve_opts* opts, const DedupParams* dd, cudaStream_t st) {
   if (!h || N < 0 || S < 1 || maxit < 0 || std::isnan(alpha) || std::isnan(tol)) return SSHOPM_EINVAL;
   if (N == 0) return SSHOPM_OK;
+  if (opts && opts->fuse_dedup == 4) {                             // records path: no raw outputs
+    if (!dd || !d_entries || !d_starts) return SSHOPM_EINVAL;
+    if (!h->L || (opts->schedule != 0 && opts->schedule != 8)) return SSHOPM_EUNSUPPORTED;
+    return solve_records(h, N, d_entries, S, d_starts, alpha, tol, maxit, opts, dd, st);
+  }
   if (!d_entries || !d_starts || !d_out_lambda || !d_out_x || !d_out_iters || !d_out_converged) return SSHOPM_EINVAL;
   if (N > (1LL << 40) / S) return SSHOPM_EUNSUPPORTED;
   const Launchers* L = h->L;
@@ -510,24 +600,34 @@ int sshopm_apply(sshopm_t h, int64_t N, const float* d_entries, const float* d_x
 }  // extern "C"
 
 namespace sshopm {
-template <int NN, bool EVEN>
-static cudaError_t launch_dedup_t(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+template <int NN, bool EVEN, bool REC>
+static cudaError_t launch_dedup_t2(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
   if (smem > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup_kernel<NN, EVEN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup_kernel<NN, EVEN, REC>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
   }
-  sshopm_dedup_kernel<NN, EVEN><<<grid, block, smem, st>>>(p);
+  sshopm_dedup_kernel<NN, EVEN, REC><<<grid, block, smem, st>>>(p);
   return cudaGetLastError();
 }
-
 template <int NN, bool EVEN>
-static cudaError_t launch_dedup128(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+static cudaError_t launch_dedup_t(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+  return p.rec ? launch_dedup_t2<NN, EVEN, true>(p, grid, block, smem, st)
+               : launch_dedup_t2<NN, EVEN, false>(p, grid, block, smem, st);
+}
+
+template <int NN, bool EVEN, bool REC>
+static cudaError_t launch_dedup128_2(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
   if (smem > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup128_kernel<NN, EVEN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(sshopm_dedup128_kernel<NN, EVEN, REC>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
   }
-  sshopm_dedup128_kernel<NN, EVEN><<<grid, block, smem, st>>>(p);
+  sshopm_dedup128_kernel<NN, EVEN, REC><<<grid, block, smem, st>>>(p);
   return cudaGetLastError();
+}
+template <int NN, bool EVEN>
+static cudaError_t launch_dedup128(const DedupParams& p, int grid, int block, int smem, cudaStream_t st) {
+  return p.rec ? launch_dedup128_2<NN, EVEN, true>(p, grid, block, smem, st)
+               : launch_dedup128_2<NN, EVEN, false>(p, grid, block, smem, st);
 }
 
 int make_dedup_params(int n, int64_t N, int S, float lam_tol, float ang_tol, int kmax, int32_t* d_count,
@@ -539,6 +639,7 @@ int make_dedup_params(int n, int64_t N, int S, float lam_tol, float ang_tol, int
   p->lambda = nullptr;
   p->x = nullptr;
   p->conv = nullptr;
+  p->rec = nullptr;
   p->out_count = d_count;
   p->out_lambda = d_olam;
   p->out_x = d_ox;
@@ -572,10 +673,11 @@ static int dedup_launch_shape(int n, int64_t N, int S, bool fast, int* grid, int
 
 int launch_dedup(int m, int n, const DedupParams& p, cudaStream_t st) {
   if (p.n_tensors == 0) return SSHOPM_OK;
-  if (!p.lambda || !p.x || !p.conv) return SSHOPM_EINVAL;
+  if (!p.rec && (!p.lambda || !p.x || !p.conv)) return SSHOPM_EINVAL;
   const int S = p.S;
-  const bool fast = (S == 128) && n <= 8 && ((uintptr_t)p.lambda % 16 == 0) && ((uintptr_t)p.x % 16 == 0) &&
-                    ((uintptr_t)p.conv % 4 == 0);
+  const bool fast = (S == 128) && n <= 8 &&
+                    (p.rec ? ((uintptr_t)p.rec % 16 == 0)
+                           : (((uintptr_t)p.lambda % 16 == 0) && ((uintptr_t)p.x % 16 == 0) && ((uintptr_t)p.conv % 4 == 0)));
   int grid, block, smem;
   int rc = dedup_launch_shape(n, p.n_tensors, S, fast, &grid, &block, &smem);
   if (rc != SSHOPM_OK) return rc;

@@ -32,7 +32,11 @@ struct DedupParams {
   long long n_tensors;
   int S, kmax;
   float lam_tol, cos_tol;  // cos(ang_tol) (may be negative)
+  const float4* rec;       // records path (sshopm_solve_rec_kernel): [N][S][rec4(n)] float4 per start,
+                           // (x_0 .. x_{n-1}, lambda if converged else NaN, 0 pad); null = the raw arrays above
 };
+// float4s per start record of the records path: lambda + n components, padded to a multiple of 4 words
+__host__ __device__ constexpr int dd_rec4(int n) { return (n + 1 + 3) / 4; }
 
 // shared-memory words per warp for S starts, dimension n
 __host__ __device__ constexpr int dedup_smem_words(int S, int n) { return S * (n + 2) + 3 * S; }
@@ -72,16 +76,33 @@ __device__ __forceinline__ float dd_norm2(const float (&x)[N]) {
 // memory): s_lam[S], s_x[S*N], s_cid[S], c_lam[S], c_rep[S], c_mult[S].  Inputs
 // are read with ld.global.cg (L2), so the routine is also safe right after
 // other lanes of the same warp wrote them (fused solve -> dedup; caller fences).
-template <int N, bool EVEN>
+template <int N, bool EVEN, bool REC = false>
 __device__ __forceinline__ void warp_dedup_tensor(const DedupParams& p, long long v, int lane, float* s_lam,
                                                   float* s_x, int* s_cid, float* c_lam, int* c_rep, int* c_mult) {
   const int S = p.S;
   const long long b = v * S;
-  for (int s = lane; s < S; s += 32) {
-    s_lam[s] = __ldcg(p.lambda + b + s);
-    s_cid[s] = __ldcg(p.conv + b + s) ? -1 : -2;
+  if constexpr (REC) {     // records: converged <=> lambda is not NaN (a converged lambda is finite)
+    constexpr int R4 = dd_rec4(N);
+    for (int s = lane; s < S; s += 32) {
+      const float4* r = p.rec + (b + s) * R4;
+      float w[4 * R4];
+#pragma unroll
+      for (int i = 0; i < R4; ++i) {
+        const float4 q = __ldcg(r + i);
+        w[4 * i] = q.x; w[4 * i + 1] = q.y; w[4 * i + 2] = q.z; w[4 * i + 3] = q.w;
+      }
+      s_lam[s] = w[N];
+      s_cid[s] = (w[N] == w[N]) ? -1 : -2;
+#pragma unroll
+      for (int j = 0; j < N; ++j) s_x[s * N + j] = w[j];
+    }
+  } else {
+    for (int s = lane; s < S; s += 32) {
+      s_lam[s] = __ldcg(p.lambda + b + s);
+      s_cid[s] = __ldcg(p.conv + b + s) ? -1 : -2;
+    }
+    for (int t = lane; t < S * N; t += 32) s_x[t] = __ldcg(p.x + b * N + t);
   }
-  for (int t = lane; t < S * N; t += 32) s_x[t] = __ldcg(p.x + b * N + t);
   __syncwarp();
 
   const float ct2 = p.cos_tol * p.cos_tol;
@@ -142,7 +163,7 @@ __device__ __forceinline__ void warp_dedup_tensor(const DedupParams& p, long lon
   __syncwarp();
 }
 
-template <int N, bool EVEN>
+template <int N, bool EVEN, bool REC = false>
 __global__ void __launch_bounds__(256) sshopm_dedup_kernel(const DedupParams p) {
   extern __shared__ float smem[];
   const int lane = threadIdx.x & 31;
@@ -156,7 +177,7 @@ __global__ void __launch_bounds__(256) sshopm_dedup_kernel(const DedupParams p) 
   int* c_mult = c_rep + S;
   const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
   for (long long v = (long long)blockIdx.x * (blockDim.x >> 5) + wib; v < p.n_tensors; v += warps)
-    warp_dedup_tensor<N, EVEN>(p, v, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
+    warp_dedup_tensor<N, EVEN, REC>(p, v, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
 }
 
 // Dedup of the tensors of listed chunks (fused solve: chunks whose completion
@@ -216,9 +237,37 @@ __device__ __forceinline__ void dedup_load(DedupRegs<N>& r, const DedupParams& p
   }
 }
 
+// records path: lane l holds starts l, l + 32, l + 64, l + 96 (coalesced record loads; start index of
+// register slot c = l + 32 c, the LANEMAJ form of dedup128_regs), one (x, lambda | NaN) record each
+template <int N>
+__device__ __forceinline__ void dedup_load_rec(DedupRegs<N>& r, const DedupParams& p, long long v, int lane) {
+  constexpr int R4 = dd_rec4(N);
+  const float4* pr = p.rec + (v * 128) * R4;
+  float w[4][4 * R4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c)
+#pragma unroll
+    for (int i = 0; i < R4; ++i) {
+      const float4 q = __ldcs(pr + (size_t)(lane + 32 * c) * R4 + i);
+      w[c][4 * i] = q.x; w[c][4 * i + 1] = q.y; w[c][4 * i + 2] = q.z; w[c][4 * i + 3] = q.w;
+    }
+  r.lam = make_float4(w[0][N], w[1][N], w[2][N], w[3][N]);
+  float xf[4 * N];
+#pragma unroll
+  for (int c = 0; c < 4; ++c)
+#pragma unroll
+    for (int j = 0; j < N; ++j) xf[c * N + j] = w[c][j];
+#pragma unroll
+  for (int i = 0; i < N; ++i) r.x[i] = make_float4(xf[4 * i], xf[4 * i + 1], xf[4 * i + 2], xf[4 * i + 3]);
+  r.conv = (w[0][N] == w[0][N] ? 0x1u : 0u) | (w[1][N] == w[1][N] ? 0x100u : 0u) | (w[2][N] == w[2][N] ? 0x10000u : 0u) |
+           (w[3][N] == w[3][N] ? 0x1000000u : 0u);
+}
+
 // Returns false (nothing written) if the tensor has more than 32 clusters.
 // stage: per-warp 128 * (N + 1) floats of shared memory when STAGE.
-template <int N, bool EVEN, bool STAGE>
+// LANEMAJ: register slot c of lane l holds start l + 32 c (records path) instead of 4 l + c; the shared-
+// memory stage then keeps x component-major (stage[128 + j * 128 + start]).
+template <int N, bool EVEN, bool STAGE, bool LANEMAJ = false>
 __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v, int lane, const DedupRegs<N>& r,
                                               float* stage) {
   constexpr int SPL = 4;
@@ -248,7 +297,15 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
 #pragma unroll
   for (int c = 0; c < SPL; ++c) un |= ((r.conv >> (8 * c)) & 0xffu) ? (1u << c) : 0u;
 #endif
-  if constexpr (STAGE) {
+  if constexpr (STAGE && LANEMAJ) {
+#pragma unroll
+    for (int c = 0; c < SPL; ++c) {
+      stage[32 * c + lane] = lam[c];
+#pragma unroll
+      for (int j = 0; j < N; ++j) stage[128 + 128 * j + 32 * c + lane] = xs[c][j];
+    }
+    __syncwarp();
+  } else if constexpr (STAGE) {
     reinterpret_cast<float4*>(stage)[lane] = r.lam;
 #pragma unroll
     for (int i = 0; i < N; ++i) reinterpret_cast<float4*>(stage + 128)[lane * N + i] = r.x[i];
@@ -263,16 +320,16 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
 #pragma unroll 1
   for (;;) {
     const int fl = __ffs(un) - 1;                    // lowest unassigned local start (-1: none)
-    const int first = __reduce_min_sync(FULL, fl >= 0 ? SPL * lane + fl : 0x7fffffff);
+    const int first = __reduce_min_sync(FULL, fl >= 0 ? (LANEMAJ ? lane + 32 * fl : SPL * lane + fl) : 0x7fffffff);
     if (first == 0x7fffffff) break;
     if (ncl == 32) return false;                     // too many clusters for the register form
     float rl, rx[N];
     if constexpr (STAGE) {
       rl = stage[first];
 #pragma unroll
-      for (int j = 0; j < N; ++j) rx[j] = stage[128 + first * N + j];
+      for (int j = 0; j < N; ++j) rx[j] = LANEMAJ ? stage[128 + 128 * j + first] : stage[128 + first * N + j];
     } else {
-      const int src = first / SPL, fc = first % SPL;
+      const int src = LANEMAJ ? (first & 31) : first / SPL, fc = LANEMAJ ? (first >> 5) : first % SPL;
       rl = __shfl_sync(FULL, (fc == 0) ? lam[0] : (fc == 1) ? lam[1] : (fc == 2) ? lam[2] : lam[3], src);
 #pragma unroll
       for (int j = 0; j < N; ++j)
@@ -356,7 +413,7 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
 // Standalone dedup for S = 128: warp per tensor, the next tensor prefetched
 // into registers while the current one is clustered; a tensor with more than
 // 32 clusters falls back to the shared-memory routine.
-template <int N, bool EVEN>
+template <int N, bool EVEN, bool REC = false>
 __global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams p) {
   extern __shared__ float smem[];
   const int lane = threadIdx.x & 31;
@@ -366,15 +423,19 @@ __global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams 
   const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
   long long v = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
   auto run = [&](const DedupRegs<N>& cur, long long t) {
-    if (!dedup128_regs<N, EVEN, true>(p, t, lane, cur, stage)) {
+    if (!dedup128_regs<N, EVEN, true, REC>(p, t, lane, cur, stage)) {
       float* s_lam = gen;
       float* s_x = s_lam + 128;
       int* s_cid = reinterpret_cast<int*>(s_x + 128 * N);
       float* c_lam = reinterpret_cast<float*>(s_cid + 128);
       int* c_rep = reinterpret_cast<int*>(c_lam + 128);
       int* c_mult = c_rep + 128;
-      warp_dedup_tensor<N, EVEN>(p, t, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
+      warp_dedup_tensor<N, EVEN, REC>(p, t, lane, s_lam, s_x, s_cid, c_lam, c_rep, c_mult);
     }
+  };
+  auto load = [&](DedupRegs<N>& r, long long t) {
+    if constexpr (REC) dedup_load_rec<N>(r, p, t, lane);
+    else dedup_load<N>(r, p, t, lane, true);
   };
 #ifndef SSHOPM_DD_TWOBUF
 #define SSHOPM_DD_TWOBUF 0   // two alternating prefetch buffers: measured slower (0.463 ms)
@@ -382,20 +443,20 @@ __global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams 
 #if SSHOPM_DD_TWOBUF
   // two register buffers used alternately (no copy of the prefetched buffer)
   DedupRegs<N> a, b;
-  if (v < p.n_tensors) dedup_load<N>(a, p, v, lane, true);
+  if (v < p.n_tensors) load(a, v);
   for (; v < p.n_tensors; v += 2 * warps) {
-    if (v + warps < p.n_tensors) dedup_load<N>(b, p, v + warps, lane, true);
+    if (v + warps < p.n_tensors) load(b, v + warps);
     run(a, v);
     if (v + warps >= p.n_tensors) break;
-    if (v + 2 * warps < p.n_tensors) dedup_load<N>(a, p, v + 2 * warps, lane, true);
+    if (v + 2 * warps < p.n_tensors) load(a, v + 2 * warps);
     run(b, v + warps);
   }
 #else
   DedupRegs<N> nx;
-  if (v < p.n_tensors) dedup_load<N>(nx, p, v, lane, true);
+  if (v < p.n_tensors) load(nx, v);
   for (; v < p.n_tensors; v += warps) {
     const DedupRegs<N> cur = nx;
-    if (v + warps < p.n_tensors) dedup_load<N>(nx, p, v + warps, lane, true);   // prefetch
+    if (v + warps < p.n_tensors) load(nx, v + warps);   // prefetch
     run(cur, v);
   }
 #endif

@@ -132,12 +132,30 @@ cudaError_t apply(long long n_items, const float4* packed, const float* x, float
 
 int wt_smem(int S) { return wt_smem_per_warp<N>(S); }
 
+cudaError_t occupancy_rec(int shift, int* bps) {
+  switch (shift) {
+    case 0: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_rec_kernel<M, N, 0>, 256, 0);
+    case 1: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_rec_kernel<M, N, 1>, 256, 0);
+    case 2: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_rec_kernel<M, N, 2>, 256, 0);
+    default: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_rec_kernel<M, N, 3>, 256, 0);
+  }
+}
+cudaError_t solve_rec(const RecParams& p, int shift, int grid, cudaStream_t st) {
+  switch (shift) {
+    case 0: sshopm_solve_rec_kernel<M, N, 0><<<grid, 256, 0, st>>>(p); break;
+    case 1: sshopm_solve_rec_kernel<M, N, 1><<<grid, 256, 0, st>>>(p); break;
+    case 2: sshopm_solve_rec_kernel<M, N, 2><<<grid, 256, 0, st>>>(p); break;
+    default: sshopm_solve_rec_kernel<M, N, 3><<<grid, 256, 0, st>>>(p); break;
+  }
+  return cudaGetLastError();
+}
+
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
                       Sh::BFORM ? 1 : 0,
                       steps_per_trip<M, N>() == 4 ? 10 : (steps_per_trip<M, N>() == 3 ? 8 : 6), 1,   // refill threshold K
                       // (swept on B200: profiles/r1/solve_variants.txt, profiles/r2/solve_variants_s6.jsonl)
-                      wt_smem, class_index, occupancy, pack, solve, classify, apply};
+                      wt_smem, class_index, occupancy, pack, solve, classify, apply, occupancy_rec, solve_rec};
 }  // namespace
 
 #define SSHOPM_CAT2(a, b, c) get_launchers_##a##_##b

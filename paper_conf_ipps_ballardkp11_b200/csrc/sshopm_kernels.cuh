@@ -1128,6 +1128,139 @@ sshopm_solve_kernel(const SolveParams p) {
 }
 
 
+// ----------------------------------------- solve kernel, schedule 8 (records) --
+// Lane-owned work units for the records path (solve -> dedup without the raw per-start arrays).  A lane
+// claims a unit of `unit` consecutive starts of one tensor (warp-aggregated atomic on p.counter), keeps the
+// tensor's coefficient rows in its registers for the whole unit and, when its item stops, takes the
+// unit's next start: the refill is one record store, one start load and a few selects (no coefficient
+// reload, no item -> (tensor, start) arithmetic).  Each item leaves one record of REC4 float4s,
+// (x_0 .. x_{n-1}, lambda if converged else NaN, 0 pad), at rec[(t * S + s) * REC4]: every store is a
+// whole 16-byte vector (one L2 transaction), and for n = 3 the record is the lane's x registers plus one
+// select.  Item indices are 32-bit (N * S < 2^32).  The per-lane arithmetic is sshopm_step, so the
+// records carry bit for bit the values of the other schedules.
+template <int N>
+constexpr int rec4() { return (N + 1 + 3) / 4; }
+
+struct RecParams {
+  const float4* packed;      // [N][PW/4] (sshopm_pack_kernel)
+  const float4* starts_n;    // [S][SST/4]
+  float4* rec;               // [N][S][REC4]
+  unsigned long long* total_iters;   // optional
+  unsigned int* counter;     // unit counter (zeroed by the pack kernel)
+  uint32_t n_units;          // N * units_per_tensor
+  uint32_t units_per_tensor, unit, S;
+  FastDiv div_upt;           // unit -> tensor
+  float alpha, tol;
+  const float* alpha_t;      // SHIFT == 3
+  int maxit, refill_k;
+};
+
+template <int M, int N, int SHIFT>
+__global__ void __launch_bounds__(256, Shape<M, N>::MINB)
+sshopm_solve_rec_kernel(const RecParams p) {
+#ifdef SSHOPM_REC_STEPS
+  constexpr int STEPS = SSHOPM_REC_STEPS;
+#else
+  constexpr int STEPS = steps_per_trip<M, N>();
+#endif
+  constexpr int SST4 = round4(N) / 4;
+  constexpr int R4 = rec4<N>();
+  constexpr int IDLE = 0x7fffffff;
+  const int lane = threadIdx.x & 31;
+  const uint32_t ltmask = lanemask_lt();
+  const uint32_t FULL = 0xffffffffu;
+  const float alpha = (SHIFT == 2) ? -p.alpha : p.alpha;
+  const float tol = p.tol;
+  const int maxit = p.maxit;
+
+  Coefs<M, N> cf;
+  float2 xs[Shape<M, N>::NX];
+#pragma unroll
+  for (int i = 0; i < Shape<M, N>::NX; ++i) xs[i] = f2(0.f, 0.f);
+  float lamp = 0.f, lam = 0.f;
+  int k = IDLE;
+  bool has = false, stop = true, conv = false;
+  uint32_t item = 0, item_end = 0;   // current item t * S + s, end of the lane's unit
+  uint32_t s = 0;                    // current start
+  float la = 0.f, ls = 1.f;
+  uint32_t it_sum = 0;
+  bool exhausted = false;
+  uint32_t k_eff = (uint32_t)p.refill_k;
+
+  for (;;) {
+    const uint32_t smask = __ballot_sync(FULL, stop);
+    if ((uint32_t)__popc(smask) >= k_eff) {
+      const bool wr = stop && has;
+      if (wr) {                                          // the finished item's record
+        float v[4 * R4];
+#pragma unroll
+        for (int j = 0; j < N; ++j) v[j] = xget<M, N>(xs, j);
+        v[N] = conv ? lam : __int_as_float(0x7fffffff);
+#pragma unroll
+        for (int j = N + 1; j < 4 * R4; ++j) v[j] = 0.f;
+        float4* r = p.rec + (size_t)item * R4;
+#pragma unroll
+        for (int i = 0; i < R4; ++i) r[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+      }
+      if (p.total_iters != nullptr) it_sum += wr ? (uint32_t)k : 0u;
+      bool ok = wr && item + 1 < item_end;               // next start of the lane's unit
+      item += ok ? 1u : 0u;
+      s += ok ? 1u : 0u;
+      const bool need = stop && !ok;                     // unit used up (or never had one)
+      const uint32_t nmask = __ballot_sync(FULL, need);
+      if (nmask != 0u && !exhausted) {                   // claim units for those lanes (one atomic per warp)
+        const uint32_t nn = __popc(nmask);
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(p.counter, nn);
+        base = __shfl_sync(FULL, base, 0);
+        if (base + nn >= p.n_units || base + nn < base) exhausted = true;
+        const uint32_t u = base + __popc(nmask & ltmask);
+        if (need && u >= base && u < p.n_units) {
+          const uint32_t t = fast_div(u, p.div_upt);
+          s = (u - t * p.units_per_tensor) * p.unit;
+          item = t * p.S + s;
+          item_end = item + min(p.unit, p.S - s);
+          cf.load(p.packed + (size_t)t * (Shape<M, N>::PW / 4));
+          if constexpr (SHIFT == 3) {
+            const float at = __ldg(p.alpha_t + t);
+            ls = at >= 0.f ? 1.f : -1.f;
+            la = fabsf(at);
+          }
+          ok = true;
+        }
+      }
+      if (ok) {
+        float v[4 * SST4];
+#pragma unroll
+        for (int i = 0; i < SST4; ++i) {
+          const float4 q4 = ldg4(p.starts_n + s * SST4 + i);
+          v[4 * i] = q4.x; v[4 * i + 1] = q4.y; v[4 * i + 2] = q4.z; v[4 * i + 3] = q4.w;
+        }
+#pragma unroll
+        for (int i = 0; i < Shape<M, N>::NX; ++i) xs[i] = f2(v[2 * i], v[2 * i + 1]);
+      }
+      k = ok ? 0 : (stop ? IDLE : k);
+      lamp = ok ? __int_as_float(0x7fffffff) : lamp;
+      has = stop ? ok : has;
+      if (exhausted) {                                   // idle lanes stay idle: count K beyond them
+        const uint32_t idle = __popc(__ballot_sync(FULL, !has));
+        if (idle == 32u) break;
+        k_eff = min(32u, idle + (uint32_t)p.refill_k);
+      }
+    }
+#pragma unroll
+    for (int rep = 0; rep < STEPS; ++rep)
+      sshopm_step<M, N, SHIFT, true>(cf, xs, lam, lamp, k, conv, stop, has, alpha, la, ls, tol, maxit);
+    __syncwarp();
+  }
+  if (p.total_iters) {
+    unsigned long long ws = it_sum;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(0xffffffffu, ws, o);
+    if (lane == 0) atomicAdd(p.total_iters, ws);
+  }
+}
+
 // ------------------------------------------------- solve kernel, schedule 6 --
 // Item per lane with a branch-free refill (opt-in; measured 1.5% slower than schedule 1 at C2 with the
 // same step, profiles/r2/solve_variants.md).  Each warp owns one chunk of

@@ -673,3 +673,70 @@ def test_classify_convex_shift_gives_maxima(dev):
     assert filled.any()
     assert not (ty == -1).any()
     assert np.mean(np.isin(ty[filled], (1, 2))) >= 0.9
+
+
+# ------------------------------------------------ records path (schedule 8) --
+def _records(dev, m, n, ent, st, alpha, tol, maxit, lt, at, kmax, **kw):
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    tot = torch.zeros(1, dtype=torch.int64, device=dev)
+    raw, dd = s.solve_dedup(e, t, alpha, tol, maxit, lt, at, kmax, records=True, total_iters=tot, **kw)
+    torch.cuda.synchronize()
+    assert raw is None
+    return [x.cpu().numpy() for x in dd], int(tot.item())
+
+
+@pytest.mark.parametrize("m,n,V,S,alpha,kmax,unit", [(4, 3, 3000, 128, 0.0, 4, 0), (4, 3, 777, 100, 0.0, 8, 7),
+                                                     (6, 3, 500, 128, 0.25, 6, 32), (3, 3, 400, 64, 1.0, 5, 1),
+                                                     (4, 6, 200, 128, 0.0, 4, 0), (8, 3, 100, 32, 0.5, 3, 5),
+                                                     (4, 3, 50, 300, 0.0, 4, 64), (4, 3, 70, 128, -0.5, 4, 200),
+                                                     (3, 2, 33, 1, 0.0, 2, 0), (4, 3, 1, 128, 0.0, 4, 3)])
+def test_records_path_equals_two_pass(dev, m, n, V, S, alpha, kmax, unit):
+    """sshopm_solve_dedup on the records path (fuse_dedup = 4: lane-owned units, 16-byte per-start records,
+    dedup reading the records) == sshopm_solve + sshopm_dedup, bit for bit, and the same iteration total."""
+    ent = syn.gen_voxels(m, n, 900, V, 1) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 1)
+    st = syn.gen_starts(S, n, 3)
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    tot = torch.zeros(1, dtype=torch.int64, device=dev)
+    raw = s.solve(e, t, alpha, 1e-6, 100, total_iters=tot)
+    da = [x.cpu().numpy() for x in s.dedup(raw[0], raw[1], raw[3], 1e-2, 0.05, kmax)]
+    db, its = _records(dev, m, n, ent, st, alpha, 1e-6, 100, 1e-2, 0.05, kmax, unit_starts=unit)
+    for a, b in zip(da, db):
+        assert np.array_equal(a, b)
+    assert its == int(tot.item())
+
+
+@pytest.mark.parametrize("mode", ["per_tensor", "auto_max", "auto_min"])
+def test_records_path_shift_modes(dev, mode):
+    """Per-tensor and automatic shifts on the records path equal the two-pass path bit for bit."""
+    m, n, V, S = 4, 3, 300, 128
+    ent = syn.gen_voxels(m, n, 50, V, 2)
+    st = syn.gen_starts(S, n, 4)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    alpha = (torch.linspace(-1.0, 1.0, V, device=dev, dtype=torch.float32) if mode == "per_tensor" else mode)
+    s = sh.Solver(m, n)
+    raw = s.solve(e, t, alpha, 1e-6, 100)
+    da = [x.cpu().numpy() for x in s.dedup(raw[0], raw[1], raw[3], 1e-2, 0.05, 4)]
+    _, db = s.solve_dedup(e, t, alpha, 1e-6, 100, 1e-2, 0.05, 4, records=True)
+    for a, b in zip(da, [x.cpu().numpy() for x in db]):
+        assert np.array_equal(a, b)
+
+
+def test_records_path_vs_oracle(dev):
+    """The records path against the FP64 oracle: on voxels whose converged flags all agree with the oracle's,
+    cluster counts, representatives and multiplicities equal oracle solve + oracle R16 dedup, and the
+    representative lambdas agree within the parity tolerance."""
+    m, n, V, S = 4, 3, 400, 128
+    ent = syn.gen_voxels(m, n, 1234, V, 5)
+    st = syn.gen_starts(S, n, 6)
+    (cnt, clam, cx, mult, rep), _ = _records(dev, m, n, ent, st, 0.0, 1e-6, 100, 1e-2, 0.05, 8)
+    olam, ox, oit, oconv = O.sshopm(ent, st, m, n, 0.0, 1e-6, 100)
+    gpu = _solve(dev, m, n, ent, st, 0.0, 1e-6, 100)
+    ocnt, olo, oxo, omo, oro = D.dedup(olam, ox, oconv, m, 1e-2, 0.05, 8)
+    same = (gpu[3].astype(bool) == oconv.astype(bool)).all(axis=1)
+    assert same.mean() > 0.95
+    assert np.array_equal(cnt[same], ocnt[same])
+    assert np.array_equal(mult[same], omo[same])
+    assert np.array_equal(rep[same], oro[same])
+    np.testing.assert_allclose(clam[same], olo[same], rtol=1e-4, atol=1e-4)
