@@ -413,8 +413,11 @@ __device__ __forceinline__ bool dedup128_regs(const DedupParams& p, long long v,
 // Standalone dedup for S = 128: warp per tensor, the next tensor prefetched
 // into registers while the current one is clustered; a tensor with more than
 // 32 clusters falls back to the shared-memory routine.
+#ifndef SSHOPM_DD_MINB
+#define SSHOPM_DD_MINB 1   // CTAs per SM the register allocation must allow (experiment knob)
+#endif
 template <int N, bool EVEN, bool REC = false>
-__global__ void __launch_bounds__(256) sshopm_dedup128_kernel(const DedupParams p) {
+__global__ void __launch_bounds__(256, SSHOPM_DD_MINB) sshopm_dedup128_kernel(const DedupParams p) {
   extern __shared__ float smem[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
