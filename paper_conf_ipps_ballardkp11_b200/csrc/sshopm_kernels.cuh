@@ -132,6 +132,11 @@ struct H43 { static constexpr bool v = (M == 4 && N == 3 && SSHOPM_43_FORM == 5)
 #define SSHOPM_GEN_TAIL 1   // other n = 3 shapes with rows of <= 64 words: scalar lambda / ||xhat||^2 / update
                             // (C3 (6,3) solve 11.85 -> 11.60 ms; (8,3) is 0.9% slower with it, so excluded)
 #endif
+#ifndef SSHOPM_HORNER3
+#define SSHOPM_HORNER3 1   // n = 3, m >= 6 shapes evaluate Eq. 6 by Horner in x0 (horner3): C3 11.61 -> 10.75 ms,
+                           // C4a 5.87 -> 5.37 ms (profiles/r2/horner3.md); (4,3) keeps form 2 (form 5 measured slower);
+                           // (5,3) keeps the monomial form (one chaotic stress lane left the parity contract)
+#endif
 #ifndef SSHOPM_X21_TAIL
 #define SSHOPM_X21_TAIL 1   // 1 (default): forms 2/3 with lambda, ||xhat||^2 and the update in scalar FP32 (C2 4.26 -> 4.22 ms)
 #endif
@@ -527,6 +532,155 @@ __device__ __forceinline__ void horner43(const Coefs<4, 3>& cf, const float2 (&x
   g2 = fmaf(t2, x0, C2);
 }
 
+// ---------------------------------------------------------------- n = 3 Horner --
+// Eq. 6 for n = 3 regrouped as a polynomial in x0 whose coefficients are forms in (x1, x2):
+//   g_j = sum_{d=0}^{D} x0^{D-d} P_{j,d},   P_{j,d} = sum_{b+c=d} B_{(D-d,b,c),j} x1^b x2^c     (D = m - 1)
+// evaluated by Horner in x0, the (x1, x2) monomials shared by the three outputs: n (Q - 1 + D) multiply-
+// adds plus Q - 3 shared products per step instead of n Q + (monomial tree) — (6,3): 93 FP32 operations
+// instead of 115 (experiment: SSHOPM_HORNER3).  B-form rows: (g0, g1) as FFMA2 on the word pairs
+// (B_{q,0}, B_{q,1}), g2 scalar.  Raw rows ((8,3)): the solver carries the multinomial weight
+// D!/(a! b! c!) by divided powers (x1^b/b!, x2^c/c!, Horner factors x0/k, D! at the end); EXACT_RAW
+// (the apply test hook) multiplies the shared monomials by the integer weights instead, which is exact
+// on small integers and has the same Horner structure.
+template <int D>
+__host__ __device__ constexpr int h3_q(int a, int b, int c) {     // lex rank of the degree-D tuple 0^a 1^b 2^c
+  int I[D > 0 ? D : 1] = {};
+  for (int t = 0; t < D; ++t) I[t] = t < a ? 0 : (t < a + b ? 1 : 2);
+  return tuple_rank(I, D, 3);
+}
+__host__ __device__ constexpr int h3_y(int b, int c) { return (b + c) * (b + c + 1) / 2 + c; }   // (b, c) -> slot
+
+template <int M, bool EXACT_RAW = false>
+__device__ __forceinline__ void horner3(const Coefs<M, 3>& cf, float x0, float x1, float x2, float& g0, float& g1,
+                                        float& g2) {
+  using S = Shape<M, 3>;
+  constexpr int D = M - 1;
+  constexpr int NY = (D + 1) * (D + 2) / 2;
+  if constexpr (S::BFORM) {
+    float y[NY];                                   // x1^b x2^c
+    y[0] = 1.f;
+    y[h3_y(1, 0)] = x1;
+    y[h3_y(0, 1)] = x2;
+    static_for<(D > 1 ? D - 1 : 0)>([&](auto dd) {
+      constexpr int d = decltype(dd)::value + 2;
+      static_for<d + 1>([&](auto bb) {
+        constexpr int b = decltype(bb)::value, c = d - b;
+        if constexpr (b > 0) y[h3_y(b, c)] = y[h3_y(b - 1, c)] * x1;
+        else y[h3_y(b, c)] = y[h3_y(b, c - 1)] * x2;
+      });
+    });
+    constexpr int base2 = 2 * S::Q;                // B_{q,2} words
+    // level 0..1: t = B_(D,0,0) x0 + B_(D-1,1,0) x1 + B_(D-1,0,1) x2
+    constexpr int q00 = h3_q<D>(D, 0, 0), q10 = h3_q<D>(D - 1, 1, 0), q01 = h3_q<D>(D - 1, 0, 1);
+    float2 t01 = __fmul2_rn(cf.template pair<2 * q10>(), bc(x1));
+    t01 = __ffma2_rn(cf.template pair<2 * q01>(), bc(x2), t01);
+    t01 = __ffma2_rn(cf.template pair<2 * q00>(), bc(x0), t01);
+    float t2 = cf.template word<base2 + q10>() * x1;
+    t2 = fmaf(cf.template word<base2 + q01>(), x2, t2);
+    t2 = fmaf(cf.template word<base2 + q00>(), x0, t2);
+    static_for<(D > 1 ? D - 1 : 0)>([&](auto dd) {
+      constexpr int d = decltype(dd)::value + 2;
+      constexpr int qa = h3_q<D>(D - d, d, 0);
+      float2 p01 = __fmul2_rn(cf.template pair<2 * qa>(), bc(y[h3_y(d, 0)]));
+      float p2 = cf.template word<base2 + qa>() * y[h3_y(d, 0)];
+      static_for<d>([&](auto cc) {
+        constexpr int c = decltype(cc)::value + 1, b = d - c;
+        constexpr int q = h3_q<D>(D - d, b, c);
+        p01 = __ffma2_rn(cf.template pair<2 * q>(), bc(y[h3_y(b, c)]), p01);
+        p2 = fmaf(cf.template word<base2 + q>(), y[h3_y(b, c)], p2);
+      });
+      t01 = __ffma2_rn(t01, bc(x0), p01);
+      t2 = fmaf(t2, x0, p2);
+    });
+    g0 = t01.x;
+    g1 = t01.y;
+    g2 = t2;
+  } else if constexpr (EXACT_RAW) {
+    // raw rows: the multinomial weight D!/((D-d)! b! c!) rides on the shared (x1, x2) monomials,
+    // z_{b,c} = w_{b,c} x1^b x2^c (integer weights: exact on small integers, one rounding more than y)
+    constexpr Tables<M, 3> T{};
+    float y[NY];
+    y[0] = 1.f;
+    y[h3_y(1, 0)] = x1;
+    y[h3_y(0, 1)] = x2;
+    static_for<(D > 1 ? D - 1 : 0)>([&](auto dd) {
+      constexpr int d = decltype(dd)::value + 2;
+      static_for<d + 1>([&](auto bb) {
+        constexpr int b = decltype(bb)::value, c = d - b;
+        if constexpr (b > 0) y[h3_y(b, c)] = y[h3_y(b - 1, c)] * x1;
+        else y[h3_y(b, c)] = y[h3_y(b, c - 1)] * x2;
+      });
+    });
+    float z[NY];
+    static_for<NY>([&](auto ii) {
+      constexpr int i = decltype(ii)::value;
+      constexpr int d = [] { int e = 0; while ((e + 1) * (e + 2) / 2 <= i) ++e; return e; }();
+      constexpr int c = i - d * (d + 1) / 2, b = d - c;
+      constexpr float w = (float)(fact(D) / (fact(D - d) * fact(b) * fact(c)));
+      if constexpr (w == 1.0f) z[i] = y[i];
+      else z[i] = y[i] * w;
+    });
+    float t[3];
+    static_for<3>([&](auto jj) {
+      constexpr int j = decltype(jj)::value;
+      float acc = cf.template word<T.q_cls[h3_q<D>(D, 0, 0)][j]>();   // weight 1 (x0^D)
+      static_for<D>([&](auto dd) {
+        constexpr int d = decltype(dd)::value + 1;
+        constexpr int qa = h3_q<D>(D - d, d, 0);
+        float p = cf.template word<T.q_cls[qa][j]>() * z[h3_y(d, 0)];
+        static_for<d>([&](auto cc) {
+          constexpr int c = decltype(cc)::value + 1, b = d - c;
+          constexpr int q = h3_q<D>(D - d, b, c);
+          p = fmaf(cf.template word<T.q_cls[q][j]>(), z[h3_y(b, c)], p);
+        });
+        acc = fmaf(acc, x0, p);
+      });
+      t[j] = acc;
+    });
+    g0 = t[0];
+    g1 = t[1];
+    g2 = t[2];
+  } else {
+    // raw rows, solver form: divided powers v_{b,c} = x1^b x2^c / (b! c!) and Horner factors x0 / k,
+    //   g_j = D! sum_d x0^{D-d}/(D-d)! sum_{b+c=d} a_{(D-d,b,c)+e_j} v_{b,c}
+    // (21 shared factors instead of 35 weight products for (8,3): C4a 5.72 -> 5.37 ms; the 1/k factors round)
+    constexpr Tables<M, 3> T{};
+    float v[NY];
+    v[0] = 1.f;
+    v[h3_y(1, 0)] = x1;
+    v[h3_y(0, 1)] = x2;
+    static_for<(D > 1 ? D - 1 : 0)>([&](auto dd) {
+      constexpr int d = decltype(dd)::value + 2;
+      static_for<d + 1>([&](auto bb) {
+        constexpr int b = decltype(bb)::value, c = d - b;
+        if constexpr (b > 0) v[h3_y(b, c)] = v[h3_y(b - 1, c)] * (x1 * (1.0f / (float)b));
+        else v[h3_y(b, c)] = v[h3_y(b, c - 1)] * (x2 * (1.0f / (float)c));
+      });
+    });
+    float t[3];
+    static_for<3>([&](auto jj) {
+      constexpr int j = decltype(jj)::value;
+      float acc = cf.template word<T.q_cls[h3_q<D>(D, 0, 0)][j]>();
+      static_for<D>([&](auto dd) {
+        constexpr int d = decltype(dd)::value + 1;      // level d: Horner factor x0 / (D - d + 1)
+        constexpr int qa = h3_q<D>(D - d, d, 0);
+        float p = cf.template word<T.q_cls[qa][j]>() * v[h3_y(d, 0)];
+        static_for<d>([&](auto cc) {
+          constexpr int c = decltype(cc)::value + 1, b = d - c;
+          constexpr int q = h3_q<D>(D - d, b, c);
+          p = fmaf(cf.template word<T.q_cls[q][j]>(), v[h3_y(b, c)], p);
+        });
+        acc = fmaf(acc, x0 * (1.0f / (float)(D - d + 1)), p);
+      });
+      t[j] = acc;
+    });
+    constexpr float DF = (float)fact(D);
+    g0 = t[0] * DF;
+    g1 = t[1] * DF;
+    g2 = t[2] * DF;
+  }
+}
+
 // (4,3), form 4: all-scalar evaluation (16 FMUL monomials, 30 FFMA, lambda as an FMA chain).
 __device__ __forceinline__ float eval43s(const Coefs<4, 3>& cf, float x0, float x1, float x2, float& g0, float& g1,
                                          float& g2) {
@@ -711,15 +865,22 @@ __device__ __forceinline__ void sshopm_step(const Coefs<M, N>& cf, float2 (&xs)[
       ++k;
     }
     return;
-  } else if constexpr (N == 3 && SSHOPM_GEN_TAIL == 1 && S::Q * N <= 64) {
-    // other n = 3 shapes: the library contraction, then lambda, ||xhat||^2 and the update in scalar FP32
-    float mq[S::Q];
-    monomials<M, N>(xs, mq);
-    float2 gp[1];
-    float g2 = 0.f;
-    cf.contract(mq, gp, g2);
+  } else if constexpr (N == 3 && ((SSHOPM_GEN_TAIL == 1 && S::Q * N <= 64) || (SSHOPM_HORNER3 && M >= 6))) {
+    // other n = 3 shapes: the library contraction (or Horner in x0, SSHOPM_HORNER3), then lambda,
+    // ||xhat||^2 and the update in scalar FP32
     const float x0 = xs[0].x, x1 = xs[0].y, x2 = xs[1].x;
-    const float g0 = gp[0].x, g1 = gp[0].y;
+    float g0, g1, g2;
+    if constexpr (SSHOPM_HORNER3 && M >= 6) {
+      horner3<M>(cf, x0, x1, x2, g0, g1, g2);
+    } else {
+      float mq[S::Q];
+      monomials<M, N>(xs, mq);
+      float2 gp[1];
+      g2 = 0.f;
+      cf.contract(mq, gp, g2);
+      g0 = gp[0].x;
+      g1 = gp[0].y;
+    }
     lam = fmaf(x2, g2, fmaf(x1, g1, x0 * g0));
     conv = fabsf(lam - lamp) <= tol * fmaxf(1.0f, fabsf(lam));
     float h0, h1, h2;
@@ -1656,7 +1817,14 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
     }
     if constexpr (X21<M, N>::v) xs[1].y = xs[0].y;
     float lam;
-    if constexpr (H43<M, N>::v) {
+    if constexpr (N == 3 && SSHOPM_HORNER3 && M >= 6) {     // the solver's Horner evaluation (raw rows: integer
+      float g0, g1, g2;                                     // weights instead of divided powers, exact on integers)
+      horner3<M, true>(cf, xs[0].x, xs[0].y, xs[1].x, g0, g1, g2);
+      lam = fmaf(xs[1].x, g2, fmaf(xs[0].y, g1, xs[0].x * g0));
+      out_g[i * N + 0] = g0;
+      out_g[i * N + 1] = g1;
+      out_g[i * N + 2] = g2;
+    } else if constexpr (H43<M, N>::v) {
       float g0, g1, g2;
       horner43(cf, xs, g0, g1, g2);
       lam = fmaf(xs[1].x, g2, fmaf(xs[0].y, g1, xs[0].x * g0));
