@@ -153,7 +153,7 @@ cudaError_t solve_rec(const RecParams& p, int shift, int grid, cudaStream_t st) 
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
                       Sh::BFORM ? 1 : 0,
-                      steps_per_trip<M, N>() == 4 ? 10 : (steps_per_trip<M, N>() == 3 ? 8 : 6), 1,   // refill threshold K
+                      steps_per_trip<M, N>() == 4 ? 10 : (steps_per_trip<M, N>() == 3 && !(N == 3 && M >= 6) ? 8 : 6), 1,   // refill threshold K
                       // (swept on B200: profiles/r1/solve_variants.txt, profiles/r2/solve_variants_s6.jsonl)
                       wt_smem, class_index, occupancy, pack, solve, classify, apply, occupancy_rec, solve_rec};
 }  // namespace

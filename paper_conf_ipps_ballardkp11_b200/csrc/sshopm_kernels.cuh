@@ -79,7 +79,8 @@ constexpr int steps_per_trip() {
 #ifdef SSHOPM_STEPS
   return SSHOPM_STEPS;
 #else
-  return (M == 4 && N == 3) ? 4 : ((binom(M + N - 2, M - 1) * N <= 30) ? 3 : 2);
+  // n = 3, m >= 6 (Horner step): 3 steps per trip (C3 10.75 -> 10.71 ms, C4a 5.37 -> 5.32 ms at K = 6)
+  return (M == 4 && N == 3) ? 4 : ((binom(M + N - 2, M - 1) * N <= 30 || (N == 3 && M >= 6)) ? 3 : 2);
 #endif
 }
 
@@ -537,7 +538,7 @@ __device__ __forceinline__ void horner43(const Coefs<4, 3>& cf, const float2 (&x
 //   g_j = sum_{d=0}^{D} x0^{D-d} P_{j,d},   P_{j,d} = sum_{b+c=d} B_{(D-d,b,c),j} x1^b x2^c     (D = m - 1)
 // evaluated by Horner in x0, the (x1, x2) monomials shared by the three outputs: n (Q - 1 + D) multiply-
 // adds plus Q - 3 shared products per step instead of n Q + (monomial tree) — (6,3): 93 FP32 operations
-// instead of 115 (experiment: SSHOPM_HORNER3).  B-form rows: (g0, g1) as FFMA2 on the word pairs
+// instead of 115 (default for n = 3, m >= 6; SSHOPM_HORNER3=0 restores the monomial form).  B-form rows: (g0, g1) as FFMA2 on the word pairs
 // (B_{q,0}, B_{q,1}), g2 scalar.  Raw rows ((8,3)): the solver carries the multinomial weight
 // D!/(a! b! c!) by divided powers (x1^b/b!, x2^c/c!, Horner factors x0/k, D! at the end); EXACT_RAW
 // (the apply test hook) multiplies the shared monomials by the integer weights instead, which is exact
