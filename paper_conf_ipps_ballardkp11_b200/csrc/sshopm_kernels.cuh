@@ -99,7 +99,8 @@ struct Shape {
 #define SSHOPM_BFORM_MAX 64
 #endif
 #ifndef SSHOPM_RAW_MINB_SMALL
-#define SSHOPM_RAW_MINB_SMALL 2
+#define SSHOPM_RAW_MINB_SMALL 3   // raw rows of <= 48 words ((8,3)): 80 registers, 3 CTAs per SM with the Horner step
+                                  // (C4a 5.32 -> 5.27 ms, no spills; (6,3) at 3 CTAs spills and is slower: 11.42 ms)
 #endif
   static constexpr bool BFORM = (Q * N <= SSHOPM_BFORM_MAX);   // (8,3) B-form (108 words, 186 regs) measured slower: 7.5 vs 6.3 ms
   static constexpr int PW_B = Q * NP * 2 + (ODD ? 2 * QP + (Q % 2) : 0);
@@ -107,7 +108,10 @@ struct Shape {
 #ifndef SSHOPM_BFORM32_MINB
 #define SSHOPM_BFORM32_MINB 4
 #endif
-  static constexpr int MINB = BFORM ? (Q * N <= 32 ? SSHOPM_BFORM32_MINB : (Q * N <= 64 ? 2 : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
+#ifndef SSHOPM_BFORM64_MINB
+#define SSHOPM_BFORM64_MINB 2
+#endif
+  static constexpr int MINB = BFORM ? (Q * N <= 32 ? SSHOPM_BFORM32_MINB : (Q * N <= 64 ? SSHOPM_BFORM64_MINB : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
 };
 
 // State layout of x (see xget below): slot of component i.
