@@ -454,8 +454,25 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
     chunk_tensors = (int)c;
     if (opts && opts->chunk_tensors > 0) chunk_tensors = opts->chunk_tensors;
   }
-  const long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
+  long long n_chunks = (N + chunk_tensors - 1) / chunk_tensors;
   if (n_chunks >= (1LL << 32) - (1LL << 20) || N >= (1LL << 32) - (1LL << 20)) return SSHOPM_EUNSUPPORTED;
+  // schedule 1 claims chunks of items: whole tensors normally; for small problems (fewer chunks than
+  // twice the resident warps) chunks of a part of a tensor, so every resident warp gets work (C1, the
+  // paper's 1024 tensors: 512 two-tensor chunks would occupy 512 of 4736 warps)
+  long long chunk_items = (long long)chunk_tensors * S;
+  bool itemch = false;                                           // launches the FUSED_MODE 4 instance
+  if (schedule == 1 && !fused) {
+    const long long warps = (long long)sms * bps * 8;
+    if (n_chunks < 2 * warps) {
+      long long ci = ((long long)N * S + 2 * warps - 1) / (2 * warps);
+      if (ci < 32) ci = 32;
+      if (ci < chunk_items) {
+        chunk_items = ci;
+        n_chunks = ((long long)N * S + ci - 1) / ci;
+        itemch = true;
+      }
+    }
+  }
   long long grid = (long long)sms * bps;
   if (schedule == 7) {
     if (grid * 8 > N) grid = (N + 7) / 8;                          // warps claim whole tensors
@@ -487,6 +504,8 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   p.n_tensors = N;
   p.n_chunks = n_chunks;
   p.chunk_tensors = chunk_tensors;
+  p.chunk_items = chunk_items;
+  p.n_items = (long long)N * S;
   p.S = S;
   p.divS = make_fastdiv((uint32_t)S);
   p.s_log2 = -1;
@@ -508,7 +527,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   p.ovf_list = ws.ovf_list;
   p.fused_regs = fregs ? 1 : 0;
   if (schedule == 7) { fused = wt_mode; smem = wt_smem; }
-  e = L->solve(p, shift, schedule == 7 ? false : wide, schedule, fused, (int)grid, smem, st);
+  e = L->solve(p, shift, schedule == 7 ? false : wide, schedule, itemch ? 4 : fused, (int)grid, smem, st);
   if (e != cudaSuccess) { release_workspace(&ws, st); return cuda_fail(e, "sshopm_solve: launch"); }
   h->launches.fetch_add(2);
   if (dd) {

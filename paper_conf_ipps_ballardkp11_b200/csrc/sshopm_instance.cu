@@ -45,6 +45,7 @@ cudaError_t occ2(int schedule, int smem, int* bps) {
 }
 template <int SH, bool W>
 cudaError_t occ1(int schedule, int fused, int smem, int* bps) {
+  if (fused == 4) return occ2<SH, W, 4>(schedule, smem, bps);   // schedule 1 with item chunks (small N)
   if (fused == 3) return occ2<SH, W, 3>(schedule, smem, bps);
   return fused == 2 ? occ2<SH, W, 2>(schedule, smem, bps) : fused == 1 ? occ2<SH, W, 1>(schedule, smem, bps)
                     : occ2<SH, W, 0>(schedule, smem, bps);
@@ -95,6 +96,7 @@ cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaS
 }
 template <int SH, bool W>
 cudaError_t solve1(const SolveParams& p, int schedule, int fused, int grid, int smem, cudaStream_t st) {
+  if (fused == 4) return solve2<SH, W, 4>(p, schedule, grid, smem, st);   // schedule 1 with item chunks (small N)
   if (fused == 3) return solve2<SH, W, 3>(p, schedule, grid, smem, st);
   return fused == 2 ? solve2<SH, W, 2>(p, schedule, grid, smem, st) : fused == 1 ? solve2<SH, W, 1>(p, schedule, grid, smem, st)
                     : solve2<SH, W, 0>(p, schedule, grid, smem, st);

@@ -985,6 +985,8 @@ struct SolveParams {
   unsigned int* ovf_count;   // chunks whose completion could not be tracked (zeroed by the pack kernel)
   unsigned int* ovf_list;    // their chunk indices -> sshopm_dedup_list_kernel
   int fused_regs;            // S == 128 with 16-byte aligned raw outputs: register-resident dedup, no staging smem
+  long long chunk_items;     // FUSED_MODE 4 (small N): items per claimed chunk (part of a tensor)
+  long long n_items;         // N * S
 };
 
 constexpr int kFusedRing = 16;   // open-chunk ring per warp (fused solve -> dedup), power of two
@@ -1016,7 +1018,8 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 template <int M, int N, int SHIFT, bool WIDE, int FUSED_MODE>
 __global__ void __launch_bounds__(256, Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
-  constexpr bool FUSED = FUSED_MODE != 0;        // 1: shared-memory dedup (any S <= 1024), 2: register dedup (S = 128)
+  constexpr bool ITEMCH = FUSED_MODE == 4;       // 4: not fused; chunks of items instead of whole tensors (small N)
+  constexpr bool FUSED = FUSED_MODE != 0 && !ITEMCH;   // 1: shared-memory dedup (any S <= 1024), 2: register dedup (S = 128)
   constexpr bool WS = FUSED_MODE == 3;           // 3: warp-specialised (a dedup warp per CTA consumes completed chunks)
   constexpr int STEPS = steps_per_trip<M, N>();        // SS-HOPM steps between refill checks
   using S = Shape<M, N>;
@@ -1088,7 +1091,7 @@ sshopm_solve_kernel(const SolveParams p) {
   }
 
   // warp-uniform chunk state
-  Idx c_vox = 0;              // first tensor of the current chunk
+  Idx c_vox = 0;              // first tensor (ITEMCH: first item) of the current chunk
   uint32_t c_next = 0, c_end = 0;
   bool exhausted = false;
 
@@ -1123,9 +1126,15 @@ sshopm_solve_kernel(const SolveParams p) {
         if (lane == 0) ch = atomicAdd(p.counter, 1u);
         ch = __shfl_sync(FULL, ch, 0);
         if ((long long)ch < p.n_chunks) {
-          n_vox = (Idx)ch * (Idx)p.chunk_tensors;
-          const long long nt = p.n_tensors - (long long)n_vox;
-          n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
+          if constexpr (ITEMCH) {                          // chunks of items (small problems)
+            n_vox = (Idx)ch * (Idx)p.chunk_items;           // first item of the chunk
+            const long long ni = p.n_items - (long long)n_vox;
+            n_end = (uint32_t)(ni < p.chunk_items ? ni : p.chunk_items);
+          } else {                                         // chunks of whole tensors
+            n_vox = (Idx)ch * (Idx)p.chunk_tensors;         // first tensor of the chunk
+            const long long nt = p.n_tensors - (long long)n_vox;
+            n_end = (uint32_t)((nt < p.chunk_tensors ? nt : p.chunk_tensors) * S_);
+          }
           if constexpr (FUSED) {
             ++claim_seq;
             const int slot = claim_seq & (kFusedRing - 1);
@@ -1164,7 +1173,8 @@ sshopm_solve_kernel(const SolveParams p) {
       const bool ok = stop && !exhausted && (cur || t < n_end);
       if (ok) {
         const Idx v0 = cur ? c_vox : n_vox;
-        item = v0 * (Idx)S_ + (Idx)t;
+        if constexpr (ITEMCH) item = v0 + (Idx)t;
+        else item = v0 * (Idx)S_ + (Idx)t;
         Idx tv;                                            // tensor of the item
         uint32_t s;                                        // its start
 #ifndef SSHOPM_ASSUME_POW2
@@ -1173,6 +1183,14 @@ sshopm_solve_kernel(const SolveParams p) {
         if (SSHOPM_ASSUME_POW2 || p.s_log2 >= 0) {         // S a power of two (the paper's 128): shift and mask
           tv = item >> p.s_log2;
           s = (uint32_t)item & p.s_mask;
+        } else if constexpr (ITEMCH) {
+          if constexpr (WIDE) {
+            tv = item / (Idx)S_;
+            s = (uint32_t)(item - tv * (Idx)S_);
+          } else {
+            tv = fast_div((uint32_t)item, p.divS);
+            s = (uint32_t)item - (uint32_t)tv * S_;
+          }
         } else {
           const uint32_t vq = fast_div(t, p.divS);
           s = t - vq * S_;

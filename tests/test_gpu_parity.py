@@ -740,3 +740,25 @@ def test_records_path_vs_oracle(dev):
     assert np.array_equal(mult[same], omo[same])
     assert np.array_equal(rep[same], oro[same])
     np.testing.assert_allclose(clam[same], olo[same], rtol=1e-4, atol=1e-4)
+
+
+@pytest.mark.parametrize("m,n,V,S,alpha", [(4, 3, 64, 128, 0.0), (4, 3, 50, 100, 0.5), (6, 3, 20, 77, 0.25),
+                                           (3, 3, 9, 33, -1.0)])
+def test_small_problem_item_chunks(dev, m, n, V, S, alpha):
+    """Small problems (fewer whole-tensor chunks than resident warps) run schedule 1 with chunks of items
+    (parts of tensors): results bit for bit those of schedule 2 (tensor per lane) and of the lean schedule,
+    including a non-power-of-two S (item -> tensor by division) and per-tensor shifts."""
+    ent = syn.gen_voxels(m, n, 77, V, 4) if m % 2 == 0 else syn.gen_uniform_tensors(m, n, V, 4)
+    st = syn.gen_starts(S, n, 5)
+    a = _solve(dev, m, n, ent, st, alpha, 1e-6, 100)
+    b = _solve(dev, m, n, ent, st, alpha, 1e-6, 100, schedule=2)
+    c = _solve(dev, m, n, ent, st, alpha, 1e-6, 100, schedule=6)
+    for x, y, z in zip(a, b, c):
+        assert np.array_equal(x, y) and np.array_equal(x, z)
+    per = torch.linspace(-0.5, 0.5, V, device=dev, dtype=torch.float32)
+    s = sh.Solver(m, n)
+    e, t = torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev)
+    p1 = [x.cpu().numpy() for x in s.solve(e, t, per, 1e-6, 100)]
+    p6 = [x.cpu().numpy() for x in s.solve(e, t, per, 1e-6, 100, schedule=6)]
+    for x, y in zip(p1, p6):
+        assert np.array_equal(x, y)
