@@ -27,6 +27,7 @@ struct Launchers {
   // records path (schedule 8, sshopm_solve_dedup with fuse_dedup = 4)
   cudaError_t (*occupancy_rec)(int shift, int* blocks_per_sm);
   cudaError_t (*solve_rec)(const RecParams& p, int shift, int grid, cudaStream_t st);
+  int solve_tpb;             // threads per CTA of the non-fused schedule-1 solve kernel (256, or 128 for (6,3))
 };
 
 }  // namespace sshopm

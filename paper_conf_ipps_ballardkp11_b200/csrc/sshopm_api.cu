@@ -461,8 +461,9 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   // paper's 1024 tensors: 512 two-tensor chunks would occupy 512 of 4736 warps)
   long long chunk_items = (long long)chunk_tensors * S;
   bool itemch = false;                                           // launches the FUSED_MODE 4 instance
+  const int wpc = (schedule == 1 && !fused) ? L->solve_tpb / 32 : 8;   // warps per solve CTA
   if (schedule == 1 && !fused) {
-    const long long warps = (long long)sms * bps * 8;
+    const long long warps = (long long)sms * bps * wpc;
     if (n_chunks < 2 * warps) {
       long long ci = ((long long)N * S + 2 * warps - 1) / (2 * warps);
       if (ci < 32) ci = 32;
@@ -477,7 +478,7 @@ static int solve_impl(sshopm_t h, int64_t N, const float* d_entries, int S, cons
   if (schedule == 7) {
     if (grid * 8 > N) grid = (N + 7) / 8;                          // warps claim whole tensors
   } else if (schedule != 2) {
-    if (grid * 8 > n_chunks) grid = (n_chunks + 7) / 8;
+    if (grid * wpc > n_chunks) grid = (n_chunks + wpc - 1) / wpc;
   } else {
     if (grid * 256 > N) grid = (N + 255) / 256;
   }

@@ -41,7 +41,8 @@ cudaError_t occ2(int schedule, int smem, int* bps) {
   }
   if (schedule == 6 && F == 0)
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_lean_kernel<M, N, SH, W>, 256, 0);
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W, F>, 256, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, sshopm_solve_kernel<M, N, SH, W, F>,
+                                                       (F == 0 || F == 4) ? Sh::TPB : 256, smem);
 }
 template <int SH, bool W>
 cudaError_t occ1(int schedule, int fused, int smem, int* bps) {
@@ -90,7 +91,7 @@ cudaError_t solve2(const SolveParams& p, int schedule, int grid, int smem, cudaS
 #ifndef SSHOPM_SOLVE_THREADS
 #define SSHOPM_SOLVE_THREADS 256
 #endif
-    sshopm_solve_kernel<M, N, SH, W, F><<<grid, SSHOPM_SOLVE_THREADS, smem, st>>>(p);
+    sshopm_solve_kernel<M, N, SH, W, F><<<grid, (F == 0 || F == 4) ? Sh::TPB : SSHOPM_SOLVE_THREADS, smem, st>>>(p);
   }
   return cudaGetLastError();
 }
@@ -157,7 +158,7 @@ const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       Sh::BFORM ? 1 : 0,
                       steps_per_trip<M, N>() == 4 ? 10 : (steps_per_trip<M, N>() == 3 && !(N == 3 && M >= 6) ? 8 : 6), 1,   // refill threshold K
                       // (swept on B200: profiles/r1/solve_variants.txt, profiles/r2/solve_variants_s6.jsonl)
-                      wt_smem, class_index, occupancy, pack, solve, classify, apply, occupancy_rec, solve_rec};
+                      wt_smem, class_index, occupancy, pack, solve, classify, apply, occupancy_rec, solve_rec, Sh::TPB};
 }  // namespace
 
 #define SSHOPM_CAT2(a, b, c) get_launchers_##a##_##b

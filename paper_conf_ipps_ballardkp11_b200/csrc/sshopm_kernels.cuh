@@ -112,6 +112,14 @@ struct Shape {
 #define SSHOPM_BFORM64_MINB 2
 #endif
   static constexpr int MINB = BFORM ? (Q * N <= 32 ? SSHOPM_BFORM32_MINB : (Q * N <= 64 ? SSHOPM_BFORM64_MINB : 1)) : (U <= 48 ? SSHOPM_RAW_MINB_SMALL : 1);
+  // threads per CTA of the non-fused schedule-1 solve kernel (knob): 128-thread CTAs for n = 3, m >= 6
+  // B-form rows fit a fifth CTA at <= 96 registers (20 instead of 16 warps per SM) but measured no faster
+  // at C3 (10.78 vs 10.70 ms), so the default stays 256
+#ifndef SSHOPM_TPB_BFORM63
+#define SSHOPM_TPB_BFORM63 256
+#endif
+  static constexpr int TPB = (N == 3 && M >= 6 && BFORM && Q * N > 32) ? SSHOPM_TPB_BFORM63 : 256;
+  static constexpr int MINB_T = TPB == 256 ? MINB : (65536 / (TPB * 96));   // <= 96 registers at 128 threads
 };
 
 // State layout of x (see xget below): slot of component i.
@@ -1016,7 +1024,8 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 // written the chunk's last item (open chunks tracked in a shared-memory ring;
 // untracked chunks go to p.ovf_list for sshopm_dedup_list_kernel).
 template <int M, int N, int SHIFT, bool WIDE, int FUSED_MODE>
-__global__ void __launch_bounds__(256, Shape<M, N>::MINB)
+__global__ void __launch_bounds__((FUSED_MODE == 0 || FUSED_MODE == 4) ? Shape<M, N>::TPB : 256,
+                                  (FUSED_MODE == 0 || FUSED_MODE == 4) ? Shape<M, N>::MINB_T : Shape<M, N>::MINB)
 sshopm_solve_kernel(const SolveParams p) {
   constexpr bool ITEMCH = FUSED_MODE == 4;       // 4: not fused; chunks of items instead of whole tensors (small N)
   constexpr bool FUSED = FUSED_MODE != 0 && !ITEMCH;   // 1: shared-memory dedup (any S <= 1024), 2: register dedup (S = 128)
