@@ -694,6 +694,118 @@ __device__ __forceinline__ void horner3(const Coefs<M, 3>& cf, float x0, float x
   }
 }
 
+// --------------------------------------------------------- any n: Horner in x0 --
+// Raw rows, any n (default for n >= 6; SSHOPM_HORNERN=0 restores the monomial form): g_j = D! sum_{d} x0^{D-d}/(D-d)! sum_{|t| = d} a_{(0^{D-d} t) + e_j} v_t
+// over tail multisets t of the variables 1..n-1 with divided powers v_t = prod x_i^{k_i} / k_i!
+// (v_t = v_{t - l} x_l / k_l, l the last index of t), Horner in x0 with factors x0 / k.
+template <int M, int N>
+struct HTab {
+  static constexpr int D = M - 1;
+  static constexpr int NT = binom(D + N - 1, D);      // tail multisets of degree 0..D over N-1 variables
+  int deg_off[D + 2];
+  int parent[NT];      // index of t minus its last element (-1 for t = {})
+  int var[NT];         // its last element l (1..N-1)
+  int mult[NT];        // multiplicity of l in t
+  int q[NT];           // degree-D multiset 0^{D-|t|} t as a Tables<M,N> q index
+  long long w[NT];     // multinomial weight D! / ((D-|t|)! prod k_i!) of x0^{D-|t|} x^t (EXACT form)
+  constexpr HTab() : deg_off(), parent(), var(), mult(), q(), w() {
+    long long fp[NT > 0 ? NT : 1] = {};   // prod k_i! of t
+    int off = 0;
+    for (int d = 0; d <= D; ++d) {
+      deg_off[d] = off;
+      int I[D > 0 ? D : 1] = {};
+      for (int i = 0; i < d; ++i) I[i] = 1;
+      const int cnt = binom(d + N - 2, d);
+      for (int c = 0; c < cnt; ++c) {
+        const int idx = off + c;
+        if (d == 0) { parent[idx] = -1; var[idx] = 0; mult[idx] = 0; }
+        else {
+          int J[D > 0 ? D : 1] = {};
+          for (int i = 0; i < d - 1; ++i) J[i] = I[i] - 1;   // tuple over {0..N-2} for ranking
+          parent[idx] = deg_off[d - 1] + tuple_rank(J, d - 1, N - 1);
+          var[idx] = I[d - 1];
+          int k = 0;
+          for (int i = 0; i < d; ++i) k += (I[i] == I[d - 1]);
+          mult[idx] = k;
+        }
+        fp[idx] = d == 0 ? 1 : fp[parent[idx]] * mult[idx];
+        w[idx] = fact(D) / (fact(D - d) * fp[idx]);
+        int K[D > 0 ? D : 1] = {};
+        for (int i = 0; i < D - d; ++i) K[i] = 0;
+        for (int i = 0; i < d; ++i) K[D - d + i] = I[i];
+        q[idx] = tuple_rank(K, D, N);
+        // next tuple over {1..N-1}
+        if (d > 0) {
+          int j = d - 1;
+          while (j >= 0 && I[j] == N - 1) --j;
+          if (j >= 0) { I[j] += 1; for (int k2 = j + 1; k2 < d; ++k2) I[k2] = I[j]; }
+        }
+      }
+      off += cnt;
+    }
+    deg_off[D + 1] = off;
+  }
+};
+
+// EXACT (the apply test hook): plain monomials times the integer weights, plain Horner in x0 (exact on
+// small integers; same structure, one weight product per tail monomial instead of the 1/k factors).
+template <int M, int N, bool EXACT = false>
+__device__ __forceinline__ void hornerN(const Coefs<M, N>& cf, const float (&x)[N], float (&g)[N]) {
+  using H = HTab<M, N>;
+  constexpr H T{};
+  constexpr Tables<M, N> TT{};
+  constexpr int D = M - 1;
+  float v[H::NT];
+  v[0] = 1.f;
+  static_for<H::NT - 1>([&](auto ii) {
+    constexpr int i = decltype(ii)::value + 1;
+    constexpr int par = T.parent[i], l = T.var[i], k = T.mult[i];
+    if constexpr (par == 0) v[i] = x[l];
+    else if constexpr (k == 1 || EXACT) v[i] = v[par] * x[l];
+    else v[i] = v[par] * (x[l] * (1.0f / (float)k));
+  });
+  if constexpr (EXACT) {
+    float z[H::NT];
+    static_for<H::NT>([&](auto ii) {
+      constexpr int i = decltype(ii)::value;
+      constexpr long long wi = H{}.w[i];
+      if constexpr (wi == 1) z[i] = v[i];
+      else z[i] = v[i] * (float)wi;
+    });
+    static_for<N>([&](auto jj) {
+      constexpr int j = decltype(jj)::value;
+      float acc = cf.template word<TT.q_cls[T.q[0]][j]>();
+      static_for<D>([&](auto dd) {
+        constexpr int d = decltype(dd)::value + 1;
+        constexpr int o = T.deg_off[d], cnt = T.deg_off[d + 1] - T.deg_off[d];
+        float p = cf.template word<TT.q_cls[T.q[o]][j]>() * z[o];
+        static_for<cnt - 1>([&](auto cc) {
+          constexpr int i = o + decltype(cc)::value + 1;
+          p = fmaf(cf.template word<TT.q_cls[T.q[i]][j]>(), z[i], p);
+        });
+        acc = fmaf(acc, x[0], p);
+      });
+      g[j] = acc;
+    });
+    return;
+  }
+  static_for<N>([&](auto jj) {
+    constexpr int j = decltype(jj)::value;
+    float acc = cf.template word<TT.q_cls[T.q[0]][j]>();
+    static_for<D>([&](auto dd) {
+      constexpr int d = decltype(dd)::value + 1;
+      constexpr int o = T.deg_off[d], cnt = T.deg_off[d + 1] - T.deg_off[d];
+      float p = cf.template word<TT.q_cls[T.q[o]][j]>() * v[o];
+      static_for<cnt - 1>([&](auto cc) {
+        constexpr int i = o + decltype(cc)::value + 1;
+        p = fmaf(cf.template word<TT.q_cls[T.q[i]][j]>(), v[i], p);
+      });
+      acc = fmaf(acc, x[0] * (1.0f / (float)(D - d + 1)), p);
+    });
+    g[j] = acc * (float)fact(D);
+  });
+}
+
 // (4,3), form 4: all-scalar evaluation (16 FMUL monomials, 30 FFMA, lambda as an FMA chain).
 __device__ __forceinline__ float eval43s(const Coefs<4, 3>& cf, float x0, float x1, float x2, float& g0, float& g1,
                                          float& g2) {
@@ -738,13 +850,26 @@ __device__ __forceinline__ float eval43n(const Coefs<4, 3>& cf, const float2 (&x
 }
 
 // g = A x^{M-1} (pairs gp, odd tail gs) and lambda = x . g
+#ifndef SSHOPM_HORNERN
+#define SSHOPM_HORNERN 1   // raw-row shapes with n >= 6 ((4,6)) evaluate Eq. 6 by hornerN: C4b 9.20 -> 8.74 ms
+#endif
 template <int M, int N>
 __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&xs)[(N + 1) / 2],
                                           float2 (&gp)[Shape<M, N>::NP > 0 ? Shape<M, N>::NP : 1], float& gs) {
   using S = Shape<M, N>;
-  float mq[S::Q];
-  monomials<M, N>(xs, mq);
-  cf.contract(mq, gp, gs);
+  if constexpr (SSHOPM_HORNERN && !S::BFORM && N >= 6) {
+    float x[N], g[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) x[i] = xget<M, N>(xs, i);
+    hornerN<M, N>(cf, x, g);
+#pragma unroll
+    for (int p = 0; p < S::NP; ++p) gp[p] = f2(g[2 * p], g[2 * p + 1]);
+    if constexpr (S::ODD) gs = g[N - 1];
+  } else {
+    float mq[S::Q];
+    monomials<M, N>(xs, mq);
+    cf.contract(mq, gp, gs);
+  }
   float lam;
   if constexpr (S::NP > 0) {
     float2 t = __fmul2_rn(xs[0], gp[0]);
@@ -1856,6 +1981,14 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
       out_g[i * N + 0] = g0;
       out_g[i * N + 1] = g1;
       out_g[i * N + 2] = g2;
+    } else if constexpr (SSHOPM_HORNERN && !Shape<M, N>::BFORM && N >= 6) {   // hornerN, integer weights
+      float xv[N], g[N];
+#pragma unroll
+      for (int j = 0; j < N; ++j) xv[j] = xget<M, N>(xs, j);
+      hornerN<M, N, true>(cf, xv, g);
+      lam = 0.f;
+#pragma unroll
+      for (int j = 0; j < N; ++j) { out_g[i * N + j] = g[j]; lam = fmaf(xv[j], g[j], lam); }
     } else if constexpr (H43<M, N>::v) {
       float g0, g1, g2;
       horner43(cf, xs, g0, g1, g2);
