@@ -583,6 +583,33 @@ __device__ __forceinline__ void horner3(const Coefs<M, 3>& cf, float x0, float x
       });
     });
     constexpr int base2 = 2 * S::Q;                // B_{q,2} words
+#ifdef SSHOPM_H3_SCALAR
+    {   // experiment: all three outputs as scalar FFMA chains (no FFMA2)
+      float tt[3];
+      static_for<3>([&](auto jj) {
+        constexpr int j = decltype(jj)::value;
+        auto W = [&](auto qq) { constexpr int q = decltype(qq)::value;
+                                return j < 2 ? cf.template word<2 * q + (j < 2 ? j : 0)>() : cf.template word<base2 + q>(); };
+        constexpr int q00 = h3_q<D>(D, 0, 0), q10 = h3_q<D>(D - 1, 1, 0), q01 = h3_q<D>(D - 1, 0, 1);
+        float t = W(std::integral_constant<int, q10>{}) * x1;
+        t = fmaf(W(std::integral_constant<int, q01>{}), x2, t);
+        t = fmaf(W(std::integral_constant<int, q00>{}), x0, t);
+        static_for<(D > 1 ? D - 1 : 0)>([&](auto dd) {
+          constexpr int d = decltype(dd)::value + 2;
+          constexpr int qa = h3_q<D>(D - d, d, 0);
+          float pp = W(std::integral_constant<int, qa>{}) * y[h3_y(d, 0)];
+          static_for<d>([&](auto cc) {
+            constexpr int c = decltype(cc)::value + 1, b = d - c;
+            pp = fmaf(W(std::integral_constant<int, h3_q<D>(D - d, b, c)>{}), y[h3_y(b, c)], pp);
+          });
+          t = fmaf(t, x0, pp);
+        });
+        tt[j] = t;
+      });
+      g0 = tt[0]; g1 = tt[1]; g2 = tt[2];
+      return;
+    }
+#endif
     // level 0..1: t = B_(D,0,0) x0 + B_(D-1,1,0) x1 + B_(D-1,0,1) x2
     constexpr int q00 = h3_q<D>(D, 0, 0), q10 = h3_q<D>(D - 1, 1, 0), q01 = h3_q<D>(D - 1, 0, 1);
     float2 t01 = __fmul2_rn(cf.template pair<2 * q10>(), bc(x1));
