@@ -17,6 +17,9 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#ifdef SSHOPM_BOUNDS_CHECK
+#include <cassert>
+#endif
 
 namespace sshopm {
 
@@ -243,6 +246,9 @@ template <int N>
 __device__ __forceinline__ void dedup_load_rec(DedupRegs<N>& r, const DedupParams& p, long long v, int lane) {
   constexpr int R4 = dd_rec4(N);
   const float4* pr = p.rec + (v * 128) * R4;
+#ifdef SSHOPM_BOUNDS_CHECK
+  assert(v < p.n_tensors && p.S == 128);
+#endif
   float w[4][4 * R4];
 #pragma unroll
   for (int c = 0; c < 4; ++c)

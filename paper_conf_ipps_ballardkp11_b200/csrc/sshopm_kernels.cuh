@@ -22,6 +22,12 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#ifdef SSHOPM_BOUNDS_CHECK
+#include <cassert>
+#define SSHOPM_CHECK(c) assert(c)   // debug builds (tools/gpu_bounds.sh): index bounds of the refill paths
+#else
+#define SSHOPM_CHECK(c) ((void)0)
+#endif
 #include <type_traits>
 #include "symm_tables.cuh"
 #include "sshopm_dedup.cuh"
@@ -1357,6 +1363,7 @@ sshopm_solve_kernel(const SolveParams p) {
           s = t - vq * S_;
           tv = v0 + (Idx)vq;
         }
+        SSHOPM_CHECK((long long)tv < p.n_tensors && s < S_ && (long long)item == (long long)tv * S_ + s);
         if constexpr (FUSED) cseq = cur ? cur_seq : claim_seq;
         if constexpr (SHIFT == 3) {
           const float at = __ldg(p.alpha_t + tv);
@@ -1543,6 +1550,7 @@ sshopm_solve_rec_kernel(const RecParams p) {
         v[N] = conv ? lam : __int_as_float(0x7fffffff);
 #pragma unroll
         for (int j = N + 1; j < 4 * R4; ++j) v[j] = 0.f;
+        SSHOPM_CHECK(item < p.n_units / p.units_per_tensor * p.S && s < p.S && item < item_end);
         float4* r = p.rec + (size_t)item * R4;
 #pragma unroll
         for (int i = 0; i < R4; ++i) r[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
@@ -1562,6 +1570,7 @@ sshopm_solve_rec_kernel(const RecParams p) {
         const uint32_t u = base + __popc(nmask & ltmask);
         if (need && u >= base && u < p.n_units) {
           const uint32_t t = fast_div(u, p.div_upt);
+          SSHOPM_CHECK(t == u / p.units_per_tensor && t < p.n_units / p.units_per_tensor);
           s = (u - t * p.units_per_tensor) * p.unit;
           item = t * p.S + s;
           item_end = item + min(p.unit, p.S - s);

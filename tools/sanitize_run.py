@@ -2,7 +2,9 @@
     compute-sanitizer --tool racecheck python tools/sanitize_run.py <case>
 cases: two_pass (C1 tensors x 128 starts, default schedule 1: pack + solve + dedup), lean (schedule 6),
 tpl (schedule 2), wt / wt_records (schedule 7 raw / fused + records-only), fused (fuse_dedup = 1: in-kernel ring + list kernel, forced overflow), blocked ((4,10),
-V = 6, schedule 5, two tensor buffers per warp), general (schedule 3), classify, run_host."""
+V = 6, schedule 5, two tensor buffers per warp), general (schedule 3), classify, run_host, records (records
+path, session 4), horner ((6,3) / (8,3) / (4,6) Horner steps and apply, session 4); two_pass at C1 size runs the
+small-problem item-chunk instance of schedule 1."""
 import os
 import sys
 
@@ -47,6 +49,21 @@ elif case == "general":
     ent = syn.gen_voxels(6, 4, 0, 16, 3)
     st = syn.gen_starts(64, 4, 1)
     sh.Solver(6, 4).solve(t(ent), t(st), 0.5, 1e-6, 200, schedule=3)
+elif case == "records":      # records path (fuse_dedup = 4): lane-owned units, 16-byte records, record dedup
+    ent = syn.gen_voxels(4, 3, 0, 1024, 0)
+    st = syn.gen_starts(128, 3, 0)
+    sh.Solver(4, 3).solve_dedup(t(ent), t(st), 0.0, 1e-6, 100, 1e-2, 0.05, 4, records=True, unit_starts=32)
+    e6 = syn.gen_voxels(4, 6, 0, 64, 2)                     # two float4 per record (n = 6), S != 128
+    s6 = syn.gen_starts(100, 6, 1)
+    sh.Solver(4, 6).solve_dedup(t(e6), t(s6), 0.0, 1e-6, 100, 1e-2, 0.05, 4, records=True, unit_starts=7)
+elif case == "horner":       # Horner evaluations: (6,3) B-form FFMA2, (8,3) raw divided powers, (4,6) hornerN
+    for (m, n, a) in ((6, 3, 0.25), (8, 3, 0.5), (4, 6, 0.0)):
+        ent = syn.gen_voxels(m, n, 0, 256, 3)
+        st = syn.gen_starts(128, n, 2)
+        s = sh.Solver(m, n)
+        lam, x, it, cv = s.solve(t(ent), t(st), a, 1e-6, 100)
+        s.dedup(lam, x, cv, 1e-2, 0.05, 4)
+        s.apply(t(ent), t(syn.gen_starts(256, n, 5)))
 elif case == "run_host":
     ent = syn.gen_voxels(4, 3, 0, 3000, 9)
     st = syn.gen_starts(128, 3, 0)
