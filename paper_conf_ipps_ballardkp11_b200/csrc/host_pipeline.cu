@@ -84,9 +84,10 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   const bool raw = h_raw_lambda || h_raw_x || h_raw_iters || h_raw_converged;
   if (raw && !(h_raw_lambda && h_raw_x && h_raw_iters && h_raw_converged)) return SSHOPM_EINVAL;
   const int n = h->n, U = h->U;
-  // default: ~16 chunks of 4K..64K tensors (C2 e2e: 16K 6.75 ms, 32K 5.88, 64K 5.65, 128K 6.33; profiles/r1/e2e_sweep.txt)
+  // default: ~16 chunks of 32K..256K tensors (round 2 sweep, profiles/r2/e2e_chunks.txt: C2 32K 5.50 / 64K 5.55 ms,
+  // C3 64K 12.85, C4a 32K 6.28 / 16K 6.66, C5 256K 39.4 / 64K 43.6; round 1: profiles/r1/e2e_sweep.txt)
   long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 16;
-  if (chunk_tensors <= 0) chunk = chunk < 4096 ? 4096 : (chunk > 65536 ? 65536 : chunk);
+  if (chunk_tensors <= 0) chunk = chunk < 32768 ? 32768 : (chunk > 262144 ? 262144 : chunk);
   if (chunk > N) chunk = N;
 
   HostCache* c;
@@ -158,6 +159,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
       else if (left > chunk + 2 * q) cn = chunk < left - 3 * q ? chunk : left - 3 * q;   // leave >= 3/4 chunk
       else if (left > 2 * q) cn = left - q;                 // ... and end on a quarter chunk
     }
+    if (cn > chunk) cn = chunk;                              // the buffers hold `chunk` tensors (q = chunk / 4 rounds down)
     if (cn < 1) cn = 1;
     if (cn > left) cn = left;
     auto mark = [&]() {

@@ -308,6 +308,23 @@ def test_run_host_matches_device_path(dev):
     assert out["total_iters"] == int(it.cpu().numpy().sum())
 
 
+@pytest.mark.parametrize("V,chunk", [(4005, 1001), (4013, 1003), (5000, 1001)])
+def test_run_host_ramp_chunk_not_multiple_of_4(dev, V, chunk):
+    """run_host's ramped chunk sizes never exceed the chunk buffers (regression: with chunk % 4 != 0 the
+    ramp-down chunk left - chunk/4 could exceed chunk by up to 3 tensors -> H2D past the buffer)."""
+    m, n = 4, 3
+    ent = syn.gen_voxels(m, n, 0, V, 9)
+    st = syn.gen_starts(32, n, 0)
+    s = sh.Solver(m, n)
+    out = s.run_host(ent, st, 0.0, 1e-6, 100, 1e-2, 0.05, 4, chunk_tensors=chunk)
+    lam, x, it, cv = s.solve(torch.from_numpy(ent).to(dev), torch.from_numpy(st).to(dev), 0.0, 1e-6, 100)
+    cnt, cl, cx, mu, rp = s.dedup(lam, x, cv, 1e-2, 0.05, 4)
+    torch.cuda.synchronize()
+    assert np.array_equal(out["count"], cnt.cpu().numpy())
+    assert np.array_equal(out["lambda"], cl.cpu().numpy())
+    assert np.array_equal(out["x"], cx.cpu().numpy())
+
+
 @pytest.mark.parametrize("schedule", [1, 2, 6])
 @pytest.mark.parametrize("V,S", [(1, 1), (3, 1), (5, 7), (40, 2), (2, 300)])
 def test_tiny_chunks(dev, V, S, schedule):
