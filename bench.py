@@ -446,7 +446,7 @@ def main():
                 "mult": torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()}
         if a.e2e_rep:                                     # representative start per cluster (diagnostic)
             outs["rep"] = torch.empty((Nloc, KMAX), dtype=torch.int32).pin_memory()
-        chunk = a.e2e_chunk or min(262144, max(32768, Nloc // 16))   # the library default (host_pipeline.cu)
+        chunk = a.e2e_chunk or min(Nloc, min(262144, max(65536, Nloc // 8)))   # the library default (host_pipeline.cu)
         solver.run_host(ent_p, st_p, cfg["alpha"], cfg["tol"], cfg["maxit"], LAM_TOL, ANG_TOL, KMAX,
                         chunk_tensors=chunk, out=outs)
         if world > 1:

@@ -1,10 +1,11 @@
 // host_pipeline.cu — sshopm_run_host: end-to-end solve + dedup on HOST buffers.
 //
-// Tensors are processed in chunks of `chunk_tensors`; chunk c runs on stream
-// c % kSlots with its own device buffers, so the host->device copy of one
-// chunk, the solve/dedup kernels of another and the device->host copy of a
-// third overlap (copy engines and SMs work concurrently).  Only the per-tensor
-// dedup records (and optionally the raw per-start outputs) come back.
+// Tensors are processed in chunks of `chunk_tensors`; chunk c uses slot c % kSlots with its own device
+// buffers and two streams: the host->device copy and the solve on a lowest-priority stream, the dedup and
+// the device->host copies on a highest-priority stream (so a finished chunk's dedup CTAs are scheduled
+// before the next chunk's pending solve CTAs; with one stream per slot the order varied from call to call:
+// C2 e2e 5.12-6.17 ms, now 5.20-5.25), so copies and kernels of different chunks overlap.  Only the
+// per-tensor dedup records (and optionally the raw per-start outputs) come back.
 //
 // Device buffers and streams are cached in the handle (HostCache) and reused
 // across calls — allocation, not transfer, would otherwise dominate; calls on
@@ -25,7 +26,9 @@ namespace sshopm {
 constexpr int kSlots = 3;
 
 struct Slot {
-  cudaStream_t st = nullptr;
+  cudaStream_t st = nullptr;       // H2D, pack + solve (lowest priority)
+  cudaStream_t hi = nullptr;       // dedup + D2H (highest priority: their CTAs go before pending solve CTAs)
+  cudaEvent_t solved = nullptr, done = nullptr;
   float *ent = nullptr, *lam = nullptr, *x = nullptr, *olam = nullptr, *ox = nullptr;
   int32_t *it = nullptr, *cnt = nullptr, *mult = nullptr, *rep = nullptr;
   uint8_t* cv = nullptr;
@@ -47,9 +50,13 @@ static void free_slots(HostCache* c) {
   for (int i = 0; i < kSlots; ++i) {
     Slot& s = c->slots[i];
     if (s.st) cudaStreamSynchronize(s.st);
+    if (s.hi) cudaStreamSynchronize(s.hi);
     cudaFree(s.ent); cudaFree(s.lam); cudaFree(s.x); cudaFree(s.olam); cudaFree(s.ox);
     cudaFree(s.it); cudaFree(s.cnt); cudaFree(s.mult); cudaFree(s.rep); cudaFree(s.cv); cudaFree(s.ws);
     if (s.st) cudaStreamDestroy(s.st);
+    if (s.hi) cudaStreamDestroy(s.hi);
+    if (s.solved) cudaEventDestroy(s.solved);
+    if (s.done) cudaEventDestroy(s.done);
     s = Slot();
   }
   cudaFree(c->d_starts);
@@ -84,10 +91,11 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
   const bool raw = h_raw_lambda || h_raw_x || h_raw_iters || h_raw_converged;
   if (raw && !(h_raw_lambda && h_raw_x && h_raw_iters && h_raw_converged)) return SSHOPM_EINVAL;
   const int n = h->n, U = h->U;
-  // default: ~16 chunks of 32K..256K tensors (round 2 sweep, profiles/r2/e2e_chunks.txt: C2 32K 5.50 / 64K 5.55 ms,
-  // C3 64K 12.85, C4a 32K 6.28 / 16K 6.66, C5 256K 39.4 / 64K 43.6; round 1: profiles/r1/e2e_sweep.txt)
-  long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 16;
-  if (chunk_tensors <= 0) chunk = chunk < 32768 ? 32768 : (chunk > 262144 ? 262144 : chunk);
+  // default: N / 8 tensors per chunk, clamped to 64K..256K (round 2 sweep with the dedup / D2H on a high-priority
+  // stream, profiles/r2/e2e_chunks.txt: C2 128K 5.15 / 64K 5.26 ms, C3 128K 11.84, C4a 64K 6.02 / 32K 6.18,
+  // C5 256K 37.6 / 128K 38.3; round 1: profiles/r1/e2e_sweep.txt)
+  long long chunk = chunk_tensors > 0 ? chunk_tensors : N / 8;
+  if (chunk_tensors <= 0) chunk = chunk < 65536 ? 65536 : (chunk > 262144 ? 262144 : chunk);
   if (chunk > N) chunk = N;
 
   HostCache* c;
@@ -124,7 +132,12 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     CK(cudaMalloc(&c->d_total, sizeof(unsigned long long)), "run_host: malloc");
     for (int i = 0; i < kSlots; ++i) {
       Slot& s = c->slots[i];
-      CK(cudaStreamCreateWithFlags(&s.st, cudaStreamNonBlocking), "run_host: stream");
+      int plo = 0, phi = 0;
+      CK(cudaDeviceGetStreamPriorityRange(&plo, &phi), "run_host: priorities");
+      CK(cudaStreamCreateWithPriority(&s.st, cudaStreamNonBlocking, plo), "run_host: stream");
+      CK(cudaStreamCreateWithPriority(&s.hi, cudaStreamNonBlocking, phi), "run_host: stream");
+      CK(cudaEventCreateWithFlags(&s.solved, cudaEventDisableTiming), "run_host: event");
+      CK(cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming), "run_host: event");
       CK(cudaMalloc(&s.ent, sizeof(float) * chunk * U), "run_host: malloc");
       CK(cudaMalloc(&s.lam, sizeof(float) * chunk * S), "run_host: malloc");
       CK(cudaMalloc(&s.x, sizeof(float) * chunk * S * n), "run_host: malloc");
@@ -170,6 +183,7 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
       tev.push_back(ev);
     };
     if (trace_path) tcn.push_back(cn);
+    CK(cudaStreamWaitEvent(s.st, s.done, 0), "run_host: wait");      // the slot's previous dedup / D2H
     mark();
     CK(cudaMemcpyAsync(s.ent, h_entries + c0 * U, sizeof(float) * cn * U, cudaMemcpyHostToDevice, s.st), "run_host: H2D");
     mark();
@@ -178,9 +192,17 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
     o.d_total_iters = c->d_total;
     o.d_workspace = s.ws;
     o.workspace_bytes = s.ws_bytes;
-    rc = sshopm_solve_dedup(h, cn, s.ent, S, c->d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, lam_tol, ang_tol,
-                            kmax, s.cnt, s.olam, s.ox, s.mult, s.rep, &o, s.st);
+    rc = sshopm_solve_ex(h, cn, s.ent, S, c->d_starts, alpha, tol, maxit, s.lam, s.x, s.it, s.cv, &o, s.st);
     if (rc != SSHOPM_OK) goto done;
+    CK(cudaEventRecord(s.solved, s.st), "run_host: event");
+    CK(cudaStreamWaitEvent(s.hi, s.solved, 0), "run_host: wait");
+    rc = sshopm_dedup(h, cn, S, s.lam, s.x, s.cv, lam_tol, ang_tol, kmax, s.cnt, s.olam, s.ox, s.mult, s.rep, s.hi);
+    if (rc != SSHOPM_OK) goto done;
+    {
+      cudaStream_t st_solve = s.st;   // the D2H copies and the trace marks follow on the dedup stream
+      s.st = s.hi;
+      s.hi = st_solve;
+    }
     mark();
     CK(cudaMemcpyAsync(h_out_count + c0, s.cnt, sizeof(int32_t) * cn, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     CK(cudaMemcpyAsync(h_out_lambda + c0 * kmax, s.olam, sizeof(float) * cn * kmax, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
@@ -195,10 +217,18 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
       CK(cudaMemcpyAsync(h_raw_converged + c0 * S, s.cv, cn * S, cudaMemcpyDeviceToHost, s.st), "run_host: D2H");
     }
     mark();
+    CK(cudaEventRecord(s.done, s.st), "run_host: event");
+    {
+      cudaStream_t st_dd = s.st;      // swap back: s.st = solve stream, s.hi = dedup stream
+      s.st = s.hi;
+      s.hi = st_dd;
+    }
   }
   const auto t_enq = std::chrono::steady_clock::now();
-  for (int i = 0; i < kSlots; ++i)
+  for (int i = 0; i < kSlots; ++i) {
     if (c->slots[i].st) CK(cudaStreamSynchronize(c->slots[i].st), "run_host: sync");
+    if (c->slots[i].hi) CK(cudaStreamSynchronize(c->slots[i].hi), "run_host: sync");
+  }
   if (trace_path && !tev.empty()) {
     const auto t_sync = std::chrono::steady_clock::now();
     auto ms = [](std::chrono::steady_clock::duration d) { return std::chrono::duration<double, std::milli>(d).count(); };
@@ -220,8 +250,10 @@ extern "C" int sshopm_run_host(sshopm_t h, int64_t N, const float* h_entries, in
 #undef CK
 done:
   if (rc != SSHOPM_OK) {
-    for (int i = 0; i < kSlots; ++i)
+    for (int i = 0; i < kSlots; ++i) {
       if (c->slots[i].st) cudaStreamSynchronize(c->slots[i].st);
+      if (c->slots[i].hi) cudaStreamSynchronize(c->slots[i].hi);
+    }
     free_slots(c);
     c->device = -1;
   }
