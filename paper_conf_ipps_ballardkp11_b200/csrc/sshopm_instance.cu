@@ -156,7 +156,9 @@ cudaError_t solve_rec(const RecParams& p, int shift, int grid, cudaStream_t st) 
 const Launchers kL = {M, N, Tables<M, N>::U, Tables<M, N>::Q, Sh::PW,
                       paper_flops_per_iter<M, N>(), executed_flops_per_iter<M, N>(),
                       Sh::BFORM ? 1 : 0,
-                      steps_per_trip<M, N>() == 4 ? 10 : (steps_per_trip<M, N>() == 3 && !(N == 3 && M >= 6) ? 8 : 6), 1,   // refill threshold K
+                      steps_per_trip<M, N>() == 4 ? 10 : (steps_per_trip<M, N>() == 3 && !(N == 3 && M >= 6) ? 8
+                                                          : (N == 3 && M >= 8 ? 4 : 6)), 1,   // refill threshold K
+                      // ((8,3) with the Horner step: K = 4, C4a 5.27 -> 5.23 ms; (6,3) keeps 6: profiles/r2/horner3.md)
                       // (swept on B200: profiles/r1/solve_variants.txt, profiles/r2/solve_variants_s6.jsonl)
                       wt_smem, class_index, occupancy, pack, solve, classify, apply, occupancy_rec, solve_rec, Sh::TPB};
 }  // namespace
