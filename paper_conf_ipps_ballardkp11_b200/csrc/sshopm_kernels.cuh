@@ -884,13 +884,16 @@ __device__ __forceinline__ float eval43n(const Coefs<4, 3>& cf, const float2 (&x
 
 // g = A x^{M-1} (pairs gp, odd tail gs) and lambda = x . g
 #ifndef SSHOPM_HORNERN
-#define SSHOPM_HORNERN 1   // raw-row shapes with n >= 6 ((4,6)) evaluate Eq. 6 by hornerN: C4b 9.20 -> 8.74 ms
+#define SSHOPM_HORNERN 1   // raw-row shapes with n >= SSHOPM_HORNERN_MIN_N evaluate Eq. 6 by hornerN: C4b 9.20 -> 8.74 ms
+#endif
+#ifndef SSHOPM_HORNERN_MIN_N
+#define SSHOPM_HORNERN_MIN_N 6
 #endif
 template <int M, int N>
 __device__ __forceinline__ float evaluate(const Coefs<M, N>& cf, const float2 (&xs)[(N + 1) / 2],
                                           float2 (&gp)[Shape<M, N>::NP > 0 ? Shape<M, N>::NP : 1], float& gs) {
   using S = Shape<M, N>;
-  if constexpr (SSHOPM_HORNERN && !S::BFORM && N >= 6) {
+  if constexpr (SSHOPM_HORNERN && !S::BFORM && N >= SSHOPM_HORNERN_MIN_N && N >= 4) {
     float x[N], g[N];
 #pragma unroll
     for (int i = 0; i < N; ++i) x[i] = xget<M, N>(xs, i);
@@ -2017,7 +2020,7 @@ sshopm_apply_kernel(long long n_items, const float4* __restrict__ packed, const 
       out_g[i * N + 0] = g0;
       out_g[i * N + 1] = g1;
       out_g[i * N + 2] = g2;
-    } else if constexpr (SSHOPM_HORNERN && !Shape<M, N>::BFORM && N >= 6) {   // hornerN, integer weights
+    } else if constexpr (SSHOPM_HORNERN && !Shape<M, N>::BFORM && N >= SSHOPM_HORNERN_MIN_N && N >= 4) {   // hornerN, integer weights
       float xv[N], g[N];
 #pragma unroll
       for (int j = 0; j < N; ++j) xv[j] = xget<M, N>(xs, j);
