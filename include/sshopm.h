@@ -108,7 +108,10 @@ int sshopm_workspace_size(sshopm_t h, int64_t N, int S, size_t* bytes);
 /* Scratch bytes of the records path (fuse_dedup = 4): N * S * 16 * ceil((n + 1) / 4). */
 int sshopm_records_size(sshopm_t h, int64_t N, int S, size_t* bytes);
 
-/* Tuning / instrumentation knobs for sshopm_solve_ex (0 / NULL = library default). */
+/* Tuning / instrumentation knobs for sshopm_solve_ex (0 / NULL = library default).  Zero-initialise the
+ * whole struct (memset) and set only the fields you need: fields are appended as the library grows
+ * (d_records, records_bytes and unit_starts were added in round 2), so a caller must be compiled against
+ * this header. */
 typedef struct {
   int refill_threshold;            /* lanes that must be idle before a warp refills (1..32); default per (m, n) */
   int ctas_per_sm;                 /* persistent CTAs per SM; default = max occupancy */
